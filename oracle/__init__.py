@@ -1,0 +1,193 @@
+"""SONG oracle — TEST INFRASTRUCTURE ONLY.
+
+A plain CPU implementation of the search SONG accelerates (Algorithm 1 of
+PAPER.md, with the §IV optimizations as switches), written from the
+paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
+product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
+no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
+R1-R8 it follows are listed in its header and in DESIGN.md §3).
+
+This module only marshals numpy arrays into ``liboracle.so`` (built by
+:func:`build`) and adds the two plain definitions the paper states in prose:
+recall and the merge of per-shard results.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from typing import Callable, Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "song_oracle.cpp")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+L2, IP, COSINE = 0, 1, 2
+METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
+
+# Mode flags (must match song_oracle.cpp's enum Flags).
+PLAIN = 0
+BOUNDED_Q = 1
+SEL = 2
+DEL = 4
+BLOOM = 8
+OPTIMIZED = BOUNDED_Q | SEL | DEL          # "hashtable-sel-del" (Fig. 7)
+OPTIMIZED_BLOOM = BOUNDED_Q | SEL | BLOOM  # "bloomfilter" (Fig. 7)
+
+_TRACE_FN = ctypes.CFUNCTYPE(
+    None, ctypes.c_void_p, ctypes.c_int64,
+    ctypes.POINTER(ctypes.c_int32), ctypes.c_int64,
+    ctypes.POINTER(ctypes.c_int32), ctypes.c_int64,
+    ctypes.POINTER(ctypes.c_int32), ctypes.c_int64)
+
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with g++ (plain -O2, no vectorisation tricks)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        cmd = ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread", "-o", _LIB, _SRC]
+        subprocess.check_call(cmd)
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_LIB)
+        P = ctypes.c_void_p
+        lib.oracle_search.restype = ctypes.c_int64
+        lib.oracle_search.argtypes = [
+            P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, ctypes.c_int32,
+            P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+            ctypes.c_int64, ctypes.c_int32, ctypes.c_int64, P, P, P,
+            ctypes.c_int32, _TRACE_FN, P]
+        lib.oracle_distance.restype = ctypes.c_float
+        lib.oracle_distance.argtypes = [P, P, ctypes.c_int32, ctypes.c_int32]
+        lib.oracle_bruteforce.restype = None
+        lib.oracle_bruteforce.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                          P, ctypes.c_int64, ctypes.c_int32, P, P, ctypes.c_int32]
+        lib.oracle_bloom_probe.restype = None
+        lib.oracle_bloom_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
+                                           ctypes.c_int64, P]
+        _lib = lib
+    return _lib
+
+
+def _f32(a):
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+def _i32(a):
+    return np.ascontiguousarray(a, dtype=np.int32)
+
+
+def _ptr(a):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def default_bloom_bits(L: int) -> int:
+    """DESIGN.md reading A11: m = 2^ceil(log2(10 * 8L)) bits."""
+    need = 10 * 8 * L
+    return 1 << int(np.ceil(np.log2(need)))
+
+
+def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OPTIMIZED,
+           bloom_bits: Optional[int] = None, entry: int = 0, max_iters: int = 1 << 40,
+           nthreads: int = 1, trace: Optional[Callable] = None):
+    """Run the oracle.  Returns (ids [nq,K] int32, dists [nq,K] f32,
+    counters [nq,2] int64 = (n_dist, n_exp), n_capped)."""
+    lib = _load()
+    data = _f32(data)
+    adj = _i32(adj)
+    queries = _f32(queries)
+    if queries.ndim == 1:
+        queries = queries[None, :]
+    n, dim = data.shape
+    degree = adj.shape[1]
+    nq = queries.shape[0]
+    assert adj.shape[0] == n and queries.shape[1] == dim
+    assert 1 <= K <= L
+    ids = np.empty((nq, K), np.int32)
+    dists = np.empty((nq, K), np.float32)
+    counters = np.empty((nq, 2), np.int64)
+    if bloom_bits is None:
+        bloom_bits = default_bloom_bits(L)
+    cb = _TRACE_FN()
+    if trace is not None:
+        def _cb(ctx, it, qp, nqq, tp, nt, vp, nv):
+            q_ids = [qp[i] for i in range(nqq)]
+            t_ids = [tp[i] for i in range(nt)]
+            v_ids = None if nv < 0 else [vp[i] for i in range(nv)]
+            trace(int(it), q_ids, t_ids, v_ids)
+        cb = _TRACE_FN(_cb)
+    capped = lib.oracle_search(_ptr(data), n, dim, _ptr(adj), degree, metric, _ptr(queries), nq,
+                               K, L, flags, int(bloom_bits), entry, int(max_iters), _ptr(ids),
+                               _ptr(dists), _ptr(counters), int(nthreads), cb, None)
+    return ids, dists, counters, int(capped)
+
+
+def distance(p, x, metric: int = L2) -> float:
+    lib = _load()
+    p = _f32(p)
+    x = _f32(x)
+    return float(lib.oracle_distance(_ptr(p), _ptr(x), p.shape[0], metric))
+
+
+def bruteforce(data, queries, K: int, metric: int = L2, nthreads: int = 1):
+    """Exact top-K under the (dist, id) order — recall ground truth B."""
+    lib = _load()
+    data = _f32(data)
+    queries = _f32(queries)
+    if queries.ndim == 1:
+        queries = queries[None, :]
+    n, dim = data.shape
+    nq = queries.shape[0]
+    ids = np.empty((nq, K), np.int32)
+    dists = np.empty((nq, K), np.float32)
+    lib.oracle_bruteforce(_ptr(data), n, dim, metric, _ptr(queries), nq, K, _ptr(ids),
+                          _ptr(dists), int(nthreads))
+    return ids, dists
+
+
+def bloom_probe(bits: int, inserted, probes):
+    lib = _load()
+    ins = _i32(inserted)
+    pr = _i32(probes)
+    out = np.empty(pr.shape[0], np.uint8)
+    lib.oracle_bloom_probe(int(bits), _ptr(ins), ins.shape[0], _ptr(pr), pr.shape[0], _ptr(out))
+    return out.astype(bool)
+
+
+def recall(found_ids, truth_ids) -> float:
+    """Mean over queries of |A ∩ B| / |B|; B = truth_ids rows."""
+    found_ids = np.asarray(found_ids)
+    truth_ids = np.asarray(truth_ids)
+    tot = 0.0
+    for a, b in zip(found_ids, truth_ids):
+        bs = set(int(x) for x in b if x >= 0)
+        if not bs:
+            continue
+        tot += len(bs & set(int(x) for x in a if x >= 0)) / len(bs)
+    return tot / max(1, len(truth_ids))
+
+
+def merge_shards(ids_per_shard, dists_per_shard, K: int):
+    """P:471 "perform graph search on each GPU and merge the results": the
+    plain definition — concatenate every shard's (dist, global id) list and keep
+    the K smallest under the (dist, id) order (R2)."""
+    ids = np.concatenate([np.asarray(x) for x in ids_per_shard], axis=1)
+    dists = np.concatenate([np.asarray(x) for x in dists_per_shard], axis=1)
+    nq = ids.shape[0]
+    out_i = np.full((nq, K), -1, np.int32)
+    out_d = np.full((nq, K), np.inf, np.float32)
+    for r in range(nq):
+        pairs = sorted((float(d), int(i)) for d, i in zip(dists[r], ids[r]) if i >= 0)
+        for j, (d, i) in enumerate(pairs[:K]):
+            out_i[r, j] = i
+            out_d[r, j] = d
+    return out_i, out_d

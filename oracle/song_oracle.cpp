@@ -1,0 +1,363 @@
+// SONG oracle — TEST INFRASTRUCTURE ONLY.
+//
+// A plain, slow, single-threaded (per query) CPU implementation of the search
+// that SONG (Zhao, Tan, Li; ICDE 2020) accelerates, written from PAPER.md.
+// Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+// --impl reference legs may load this library.  The product path
+// (paper_conf_icde_zhaotl20_b200/) never links, imports or calls it, and it
+// shares no header, helper or constant table with the CUDA path.
+//
+// Citations: "P:<line>" = /root/reference/PAPER.md line.
+//   Algorithm 1 (best-first search)
+//   bounded priority queue, Observation 1    P:413-421  (§IV-C)
+//   selected insertion                       P:425-431  (§IV-D)
+//   visited deletion                         P:433-437  (§IV-E)
+//   Bloom-filter visited set                 P:283      (§IV-B)
+//   distance measures                        P:461      (§VI)
+//
+// Readings of the paper adopted here (all listed in DESIGN.md §3):
+//   R1 topk is bounded at L = queue_len (Fig. 1 iteration 4 evicts vertex 1).
+//   R2 every comparison uses the total order key(v) = (dist(p,v), v).
+//   R3 selection applies only when |topk| = L (Fig. 4(b) iteration 1 admits 5).
+//   R4 q capacity is exactly L (reproduces Fig. 1 and Fig. 4(c)).
+//   R5 the entry vertex is a parameter (default id 0).
+//   R6 -1 entries of an adjacency row are padding; a repeated id in one row is
+//      located once (first occurrence).
+//   R7 distances: squared L2; -<p,x>; 1 - cos (zero norm -> 1); accumulated in
+//      fp64 in dimension order, rounded once to fp32; -0.0 canonicalised to +0.0.
+//   R8 Bloom filter: k = 7 bits per id by double hashing
+//      bit_i = (h1 + i*h2) mod m, h1 = fmix32(id), h2 = fmix32(id ^ 0x5bd1e995) | 1,
+//      fmix32 = MurmurHash3's 32-bit finaliser.  No deletion.
+//
+// Parity status: every function below is pinned by tests/test_oracle_*.py
+// (Fig. 1 / Fig. 4(c) traces, plain == optimized equivalence, brute-force
+// exactness, greedy special case, invariants, Bloom FPR).  Nothing is
+// "parity unpinned".
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <set>
+#include <thread>
+#include <unordered_set>
+#include <vector>
+
+namespace {
+
+enum Metric { ORACLE_L2 = 0, ORACLE_IP = 1, ORACLE_COSINE = 2 };
+
+// Mode flags.  ORACLE_PLAIN (= 0) is Algorithm 1 literally: unbounded q,
+// exact visited set never deleted from, topk bounded at L (R1).
+enum Flags {
+  ORACLE_BOUNDED_Q = 1,  // §IV-C: q keeps at most L entries
+  ORACLE_SEL = 2,        // §IV-D: selected insertion
+  ORACLE_DEL = 4,        // §IV-E: visited deletion
+  ORACLE_BLOOM = 8,      // §IV-B: visited is a Bloom filter (no deletion)
+};
+
+struct Key {
+  float dist;
+  int32_t id;
+};
+
+// R2: lexicographic (dist, id).
+bool operator<(const Key& a, const Key& b) {
+  if (a.dist < b.dist) return true;
+  if (b.dist < a.dist) return false;
+  return a.id < b.id;
+}
+
+// R7: the distance of §VI, accumulated in fp64 in index order.
+float distance(const float* p, const float* x, int dim, int metric) {
+  double out;
+  if (metric == ORACLE_L2) {
+    double acc = 0.0;
+    for (int i = 0; i < dim; ++i) {
+      double t = (double)p[i] - (double)x[i];
+      acc += t * t;
+    }
+    out = acc;
+  } else if (metric == ORACLE_IP) {
+    double acc = 0.0;
+    for (int i = 0; i < dim; ++i) acc += (double)p[i] * (double)x[i];
+    out = -acc;
+  } else {
+    double dot = 0.0, np = 0.0, nx = 0.0;
+    for (int i = 0; i < dim; ++i) {
+      dot += (double)p[i] * (double)x[i];
+      np += (double)p[i] * (double)p[i];
+      nx += (double)x[i] * (double)x[i];
+    }
+    if (np == 0.0 || nx == 0.0)
+      out = 1.0;
+    else
+      out = 1.0 - dot / (std::sqrt(np) * std::sqrt(nx));
+  }
+  float f = (float)out;
+  if (f == 0.0f) f = 0.0f;  // -0.0 -> +0.0
+  return f;
+}
+
+uint32_t fmix32(uint32_t h) {
+  h ^= h >> 16;
+  h *= 0x85ebca6bu;
+  h ^= h >> 13;
+  h *= 0xc2b2ae35u;
+  h ^= h >> 16;
+  return h;
+}
+
+// R8: the Bloom filter of §IV-B.
+struct Bloom {
+  std::vector<uint32_t> words;
+  uint64_t m;  // number of bits
+  explicit Bloom(uint64_t bits) : words((bits + 31) / 32, 0u), m(bits) {}
+  uint64_t bit(int32_t id, int i) const {
+    uint32_t h1 = fmix32((uint32_t)id);
+    uint32_t h2 = fmix32((uint32_t)id ^ 0x5bd1e995u) | 1u;
+    uint32_t h = h1 + (uint32_t)i * h2;  // 32-bit wrap-around
+    return (uint64_t)h % m;
+  }
+  bool contains(int32_t id) const {
+    for (int i = 0; i < 7; ++i) {
+      uint64_t b = bit(id, i);
+      if (!((words[b >> 5] >> (b & 31)) & 1u)) return false;
+    }
+    return true;
+  }
+  void insert(int32_t id) {
+    for (int i = 0; i < 7; ++i) {
+      uint64_t b = bit(id, i);
+      words[b >> 5] |= 1u << (b & 31);
+    }
+  }
+};
+
+// The visited set: an exact hash set, or a Bloom filter.
+struct Visited {
+  bool bloom;
+  std::unordered_set<int32_t> exact;
+  Bloom filter;
+  Visited(bool use_bloom, uint64_t bloom_bits)
+      : bloom(use_bloom), filter(use_bloom ? bloom_bits : 1) {}
+  bool contains(int32_t v) const { return bloom ? filter.contains(v) : exact.count(v) != 0; }
+  void insert(int32_t v) {
+    if (bloom)
+      filter.insert(v);
+    else
+      exact.insert(v);
+  }
+  void erase(int32_t v) {
+    if (!bloom) exact.erase(v);  // a Bloom filter cannot delete
+  }
+};
+
+typedef void (*trace_fn)(void* ctx, int64_t iteration, const int32_t* q_ids, int64_t nq,
+                         const int32_t* topk_ids, int64_t ntopk, const int32_t* visited_ids,
+                         int64_t nvisited);
+
+void emit_trace(trace_fn cb, void* ctx, int64_t it, const std::set<Key>& q,
+                const std::set<Key>& topk, const Visited& vis) {
+  if (!cb) return;
+  std::vector<int32_t> qi, ti, vi;
+  for (const Key& k : q) qi.push_back(k.id);
+  for (const Key& k : topk) ti.push_back(k.id);
+  int64_t nv = -1;  // a Bloom filter cannot be enumerated
+  if (!vis.bloom) {
+    vi.assign(vis.exact.begin(), vis.exact.end());
+    std::sort(vi.begin(), vi.end());
+    nv = (int64_t)vi.size();
+  }
+  cb(ctx, it, qi.data(), (int64_t)qi.size(), ti.data(), (int64_t)ti.size(), vi.data(), nv);
+}
+
+struct Problem {
+  const float* data;
+  int64_t n;
+  int dim;
+  const int32_t* adj;
+  int degree;
+  int metric;
+  int K, L, flags, entry;
+  uint64_t bloom_bits;
+  int64_t max_iters;
+};
+
+// Algorithm 1 with the optimizations of §IV switched by flags.
+// Step numbers refer to SURVEY.md §8(c) "Optimized mode, step by step".
+// Returns 0, or 1 if the iteration cap was reached.
+int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_out,
+               int64_t* counters, trace_fn cb, void* ctx) {
+  const int L = P.L;
+  const bool bounded = P.flags & ORACLE_BOUNDED_Q;
+  const bool sel = P.flags & ORACLE_SEL;
+  const bool del = P.flags & ORACLE_DEL;
+  Visited visited((P.flags & ORACLE_BLOOM) != 0, P.bloom_bits);
+  std::set<Key> q;     // min-priority queue (begin() = min, prev(end()) = max)
+  std::set<Key> topk;  // bounded max-priority queue (R1)
+  int64_t n_dist = 0, n_exp = 0;
+  int status = 0;
+
+  // Step 1 — Alg. 1 line 1: q and visited start with the starting point.
+  const int32_t e = P.entry;
+  q.insert(Key{distance(p, P.data + (int64_t)e * P.dim, P.dim, P.metric), e});
+  visited.insert(e);
+  n_dist = 1;
+  emit_trace(cb, ctx, 0, q, topk, visited);
+
+  std::vector<int32_t> cand;
+  int64_t it = 0;
+  // Step 2 — Alg. 1 line 2.
+  while (!q.empty()) {
+    if (it >= P.max_iters) {
+      status = 1;
+      break;
+    }
+    ++it;
+    // 2.1 — line 3: pop the minimum of q.
+    Key now = *q.begin();
+    q.erase(q.begin());
+    // 2.2 — lines 4-5: stop when topk is full and its max is better than now.
+    if ((int)topk.size() == L && *std::prev(topk.end()) < now) break;
+    // 2.3 — line 7 (+R1): push into topk; evict the max beyond L; [del] erase it
+    // from visited ("when the topk is updated, the popped-out vertex can
+    // also be deleted").
+    topk.insert(now);
+    if ((int)topk.size() > L) {
+      Key y = *std::prev(topk.end());
+      topk.erase(std::prev(topk.end()));
+      if (del) visited.erase(y.id);
+    }
+    // 2.4 — candidate locating (§V): unvisited neighbours, row order,
+    // skipping padding and repeats (R6).
+    cand.clear();
+    const int32_t* row = P.adj + (int64_t)now.id * P.degree;
+    for (int j = 0; j < P.degree; ++j) {
+      int32_t v = row[j];
+      if (v < 0) continue;
+      if (visited.contains(v)) continue;
+      if (std::find(cand.begin(), cand.end(), v) != cand.end()) continue;
+      cand.push_back(v);
+    }
+    // 2.5 — bulk distance computation (§VI).
+    std::vector<Key> ck;
+    ck.reserve(cand.size());
+    for (int32_t v : cand) ck.push_back(Key{distance(p, P.data + (int64_t)v * P.dim, P.dim, P.metric), v});
+    n_dist += (int64_t)cand.size();
+    n_exp += 1;
+    // 2.6 — maintenance, lines 12-13 with §IV-C/D/E.
+    for (const Key& k : ck) {
+      // [sel] P:429: filtered when topk is full and k is worse than all of it (R3).
+      if (sel && (int)topk.size() == L && *std::prev(topk.end()) < k) continue;
+      visited.insert(k.id);
+      q.insert(k);
+      // [bounded] P:421: pop the worst once q grows past L (R4); [del] P:435.
+      if (bounded && (int)q.size() > L) {
+        Key w = *std::prev(q.end());
+        q.erase(std::prev(q.end()));
+        if (del) visited.erase(w.id);
+      }
+    }
+    emit_trace(cb, ctx, it, q, topk, visited);
+  }
+
+  // Step 3 — line 17: the first K of topk in ascending key order, padded.
+  int i = 0;
+  for (const Key& k : topk) {
+    if (i >= P.K) break;
+    ids_out[i] = k.id;
+    dists_out[i] = k.dist;
+    ++i;
+  }
+  for (; i < P.K; ++i) {
+    ids_out[i] = -1;
+    dists_out[i] = INFINITY;
+  }
+  if (counters) {
+    counters[0] = n_dist;
+    counters[1] = n_exp;
+  }
+  return status;
+}
+
+}  // namespace
+
+extern "C" {
+
+// Search nq queries.  All pointers are host pointers; layouts are row-major:
+// data [n][dim] fp32, adj [n][degree] int32 (-1 = padding), queries [nq][dim],
+// ids/dists [nq][K], counters [nq][2] = (distance computations, expansions)
+// or NULL.  nthreads > 1 partitions the queries over std::threads (no trace).
+// Returns the number of queries that hit max_iters (0 = all finished).
+int64_t oracle_search(const float* data, int64_t n, int32_t dim, const int32_t* adj,
+                      int32_t degree, int32_t metric, const float* queries, int64_t nq,
+                      int32_t K, int32_t L, int32_t flags, int64_t bloom_bits, int32_t entry,
+                      int64_t max_iters, int32_t* ids, float* dists, int64_t* counters,
+                      int32_t nthreads, trace_fn cb, void* ctx) {
+  Problem P{data, n, dim, adj, degree, metric, K, L, flags, entry, (uint64_t)bloom_bits, max_iters};
+  if (nthreads <= 1 || cb) {
+    int64_t fails = 0;
+    for (int64_t i = 0; i < nq; ++i)
+      fails += search_one(P, queries + i * dim, ids + i * K, dists + i * K,
+                          counters ? counters + 2 * i : nullptr, cb, ctx);
+    return fails;
+  }
+  std::vector<std::thread> pool;
+  std::vector<int64_t> fails(nthreads, 0);
+  for (int t = 0; t < nthreads; ++t) {
+    pool.emplace_back([&, t]() {
+      for (int64_t i = t; i < nq; i += nthreads)
+        fails[t] += search_one(P, queries + i * dim, ids + i * K, dists + i * K,
+                               counters ? counters + 2 * i : nullptr, nullptr, nullptr);
+    });
+  }
+  for (auto& th : pool) th.join();
+  int64_t total = 0;
+  for (int64_t f : fails) total += f;
+  return total;
+}
+
+// The distance of §VI for one pair (exposed so tests can pin R7 directly).
+float oracle_distance(const float* p, const float* x, int32_t dim, int32_t metric) {
+  return distance(p, x, dim, metric);
+}
+
+// Exact top-K by scanning every point under the same key order (R2).  This is
+// the ground truth B of the recall definition on small inputs.
+void oracle_bruteforce(const float* data, int64_t n, int32_t dim, int32_t metric,
+                       const float* queries, int64_t nq, int32_t K, int32_t* ids,
+                       float* dists, int32_t nthreads) {
+  auto one = [&](int64_t qi) {
+    std::vector<Key> all((size_t)n);
+    for (int64_t v = 0; v < n; ++v)
+      all[v] = Key{distance(queries + qi * dim, data + v * dim, dim, metric), (int32_t)v};
+    int64_t k = std::min<int64_t>(K, n);
+    std::partial_sort(all.begin(), all.begin() + k, all.end());
+    for (int64_t i = 0; i < K; ++i) {
+      ids[qi * K + i] = i < k ? all[i].id : -1;
+      dists[qi * K + i] = i < k ? all[i].dist : INFINITY;
+    }
+  };
+  if (nthreads <= 1) {
+    for (int64_t i = 0; i < nq; ++i) one(i);
+    return;
+  }
+  std::vector<std::thread> pool;
+  for (int t = 0; t < nthreads; ++t)
+    pool.emplace_back([&, t]() {
+      for (int64_t i = t; i < nq; i += nthreads) one(i);
+    });
+  for (auto& th : pool) th.join();
+}
+
+// Bloom filter probe for tests of §IV-B: inserts ins[0..nins), then
+// writes 1/0 membership of probe[0..nprobe) to out.
+void oracle_bloom_probe(int64_t bits, const int32_t* ins, int64_t nins, const int32_t* probe,
+                        int64_t nprobe, uint8_t* out) {
+  Bloom b((uint64_t)bits);
+  for (int64_t i = 0; i < nins; ++i) b.insert(ins[i]);
+  for (int64_t i = 0; i < nprobe; ++i) out[i] = b.contains(probe[i]) ? 1 : 0;
+}
+
+}  // extern "C"
