@@ -1,0 +1,169 @@
+/* song.h — C ABI of the B200-native SONG search library (libsong.so).
+ *
+ * SONG: Approximate Nearest Neighbor Search on GPU (Zhao, Tan, Li; ICDE 2020).
+ * "P:<n>" cites /root/reference/PAPER.md line n.
+ *
+ * The library runs the paper's batched best-first graph search (Algorithm 1,
+ * P:41-49) decoupled into candidate locating (§V), bulk distance
+ * computation (§VI) and data-structure maintenance (§IV)
+ * with a bounded priority queue (§IV-C), selected insertion (§IV-D,
+ * P:425-431), visited deletion (§IV-E) and a shared-memory
+ * open-addressing hash or Bloom-filter visited set.  Every
+ * step runs in sm_100a kernels; there is no CPU fallback.
+ *
+ * Conventions for every entry point:
+ *  - returns SONG_OK (0) on success or a negative song_status;
+ *    song_last_error() then holds a thread-local message;
+ *  - "host" pointers are ordinary CPU memory (pinned or pageable);
+ *    "device" pointers are CUDA global memory on the index's device;
+ *  - all matrices are dense row-major; ids are int32, vectors fp32;
+ *  - the library never takes ownership of caller buffers.
+ *
+ * Semantics (DESIGN.md §3 lists every reading of the paper):
+ *  - entry vertex = params.entry (default 0; "default starting point");
+ *  - adjacency entries lie in [-1, n); -1 is padding (fixed-degree rows);
+ *  - distances: SONG_L2 = squared Euclidean, SONG_IP = -<q,x>,
+ *    SONG_COSINE = 1 - <q,x>/(|q||x|); zero-norm vectors give 1;
+ *  - ties are broken by id: every order is on the key (dist, id);
+ *  - outputs are the first K of topk in ascending (dist, id) order; if fewer
+ *    than K vertices are reached, the rest is (-1, +INF) (Alg. 1 line 17);
+ *  - q and topk both hold at most queue_len = L >= K entries (readings A1, A2).
+ */
+#ifndef SONG_H_
+#define SONG_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct song_index song_index; /* opaque; owns its device copies */
+
+typedef enum { SONG_L2 = 0, SONG_IP = 1, SONG_COSINE = 2 } song_metric;
+
+typedef enum {
+  SONG_OK = 0,
+  SONG_EINVAL = -1,       /* bad argument: NULL, sizes < 1, K > queue_len, id out of
+                             range, non-finite input value */
+  SONG_ENOMEM = -2,       /* device or host allocation failed */
+  SONG_ECUDA = -3,        /* a CUDA runtime call or kernel failed */
+  SONG_EUNSUPPORTED = -4, /* a size above the compiled maxima (degree > 32,
+                             dim > 1024, queue_len > SONG_MAX_QUEUE_LEN,
+                             shared-memory budget exceeded) */
+  SONG_EITERCAP = -5      /* a query reached params.max_iters expansions */
+} song_status;
+
+typedef enum {
+  SONG_VISITED_HASH = 0,  /* open addressing, selected insertion + visited deletion
+                             ("hashtable-sel-del", Fig. 7) */
+  SONG_VISITED_BLOOM = 1  /* Bloom filter, selected insertion, no deletion
+                             ("bloomfilter") */
+} song_visited_kind;
+
+#define SONG_MAX_DEGREE 32
+#define SONG_MAX_DIM 1024
+#define SONG_MAX_QUEUE_LEN 2048
+
+typedef struct song_search_params {
+  int32_t K;               /* results per query, 1 <= K <= queue_len */
+  int32_t queue_len;       /* L: capacity of q and of topk (§IV-C) */
+  int32_t visited;         /* song_visited_kind */
+  int32_t bloom_log2_bits; /* Bloom size m = 2^bloom_log2_bits bits; 0 = default
+                              2^ceil(log2(80 L)) (reading A11) */
+  int32_t entry;           /* starting vertex id, 0 <= entry < n */
+  int32_t max_iters;       /* expansion cap per query (0 = 1<<30); a query that
+                              reaches it is flagged, see song_search_ex */
+  int32_t warps_per_block; /* launch shape: 0 = library default */
+  int32_t blocks_per_sm;   /* launch shape: 0 = as many as fit */
+  int32_t id_offset;       /* added to every returned id (dataset sharding, P:471:
+                              shard-local ids become global ids); default 0 */
+  int32_t reserved;        /* must be 0 */
+} song_search_params;
+
+typedef struct song_index_info {
+  int64_t n;               /* points */
+  int32_t dim;             /* dimensions */
+  int32_t dim_padded;      /* row stride in floats (multiple of 4: 16 B rows) */
+  int32_t degree;          /* adjacency slots per vertex */
+  int32_t metric;          /* song_metric */
+  int64_t vector_bytes;    /* n * dim_padded * 4 */
+  int64_t graph_bytes;     /* n * degree * 4 (Table III) */
+  int32_t device;          /* CUDA device ordinal */
+  int32_t num_sms;         /* SMs on that device */
+} song_index_info;
+
+/* Fill p with the library defaults for (K, queue_len). Never fails. */
+void song_default_params(song_search_params* p, int32_t K, int32_t queue_len);
+
+/* Create an index on the current CUDA device from HOST arrays (§IV-A, P:267,
+ * graph and data are persisted in global memory before any query).
+ *   vectors   [n][dim] fp32, host; copied (rows padded to 16 B; for
+ *             SONG_COSINE rows are L2-normalised on the device).
+ *   adjacency [n][degree] int32, host; copied.  Entries in [-1, n).
+ *   out       receives the handle; *out is NULL on error.
+ * Errors: SONG_EINVAL (NULL, n < 1, dim < 1, degree < 1, id out of range,
+ * non-finite vector value), SONG_EUNSUPPORTED (degree > 32, dim > 1024),
+ * SONG_ENOMEM, SONG_ECUDA. */
+int song_index_create(const float* vectors, int64_t n, int32_t dim,
+                      const int32_t* adjacency, int32_t degree, song_metric metric,
+                      song_index** out);
+
+/* As song_index_create, but vectors and adjacency are DEVICE pointers on the
+ * current device (validated on the device); stream is a cudaStream_t or NULL
+ * (legacy default stream).  The call returns after the copies complete. */
+int song_index_create_device(const float* vectors, int64_t n, int32_t dim,
+                             const int32_t* adjacency, int32_t degree, song_metric metric,
+                             void* stream, song_index** out);
+
+/* Release the index and its device memory.  NULL is a no-op (returns 0). */
+int song_index_destroy(song_index* idx);
+
+int song_index_get_info(const song_index* idx, song_index_info* info);
+
+/* Search nq queries with HOST buffers (Alg. 1 over a batch); blocking.
+ *   queries   [nq][dim] fp32 host; ids_out [nq][K] int32 host;
+ *   dists_out [nq][K] fp32 host.  Uses song_default_params(K, queue_len).
+ * The HtoD copy of the queries, the kernel and the DtoH copy of the results all
+ * happen inside this call (Fig. 10's HtoD / kernel / DtoH).
+ * Errors: SONG_EINVAL (NULL, nq < 1, K < 1, queue_len < K, non-finite query),
+ * SONG_EUNSUPPORTED (queue_len too large), SONG_EITERCAP, SONG_ECUDA. */
+int song_search(song_index* idx, const float* queries, int64_t nq, int32_t K,
+                int32_t queue_len, int32_t* ids_out, float* dists_out);
+
+/* Search with DEVICE buffers on a caller stream; asynchronous (returns after
+ * enqueueing).  counters_out, if not NULL, receives [nq][2] int32
+ * (distance computations, expansions) per query — the algorithmic work that
+ * defines the roofline bytes.  A query that hits max_iters or has a
+ * non-finite value gets ids -1; song_index_last_status() reports it.
+ * Errors detectable before launch: SONG_EINVAL, SONG_EUNSUPPORTED, SONG_ECUDA. */
+int song_search_ex(song_index* idx, const song_search_params* params,
+                   const float* queries, int64_t nq, int32_t* ids_out, float* dists_out,
+                   int32_t* counters_out, void* stream);
+
+/* Synchronise the index's last stream and return the sticky status of the
+ * searches since the previous call (SONG_OK, SONG_EINVAL for a non-finite
+ * query, SONG_EITERCAP); clears it. */
+int song_index_last_status(song_index* idx);
+
+/* G-way merge of per-shard results ("perform graph search on each GPU
+ * and merge the results").  DEVICE buffers:
+ *   ids_in [G][nq][Kin] int32 global ids, dists_in [G][nq][Kin] fp32, each row
+ *   sorted ascending by (dist, id), -1 padded;
+ *   ids_out [nq][K], dists_out [nq][K]: the K smallest (dist, id) keys.
+ * Asynchronous on stream.  Errors: SONG_EINVAL, SONG_EUNSUPPORTED (K > 1024). */
+int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,
+                    int32_t Kin, int32_t K, int32_t* ids_out, float* dists_out,
+                    void* stream);
+
+/* Thread-local message of the last failing call ("" if none). */
+const char* song_last_error(void);
+
+/* Library version string, e.g. "song-b200 0.1 sm_100a". */
+const char* song_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SONG_H_ */

@@ -1,0 +1,449 @@
+// song_api.cu — the C ABI of include/song.h over the sm_100a kernels.
+//
+// Index layout in HBM: vectors [n][dpad] fp32 with dpad =
+// round_up(dim, 4) so every row starts on a 16 B boundary (LDG.128 gathers);
+// adjacency [n][degree] int32, -1 padded (fixed-degree storage).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "merge_kernel.cuh"
+#include "search_kernel.cuh"
+#include "song.h"
+
+struct song_index {
+  int device = 0;
+  int num_sms = 0;
+  int64_t n = 0;
+  int dim = 0, dpad = 0, degree = 0, metric = 0;
+  float* d_data = nullptr;
+  int32_t* d_adj = nullptr;
+  unsigned* d_ticket = nullptr;
+  int* d_status = nullptr;
+  cudaStream_t stream = nullptr;       // owned; used by song_search
+  cudaStream_t last_stream = nullptr;  // stream of the last search
+  // scratch for the host-buffer entry point
+  float* d_q = nullptr;
+  int32_t* d_ids = nullptr;
+  float* d_dists = nullptr;
+  size_t cap_q = 0, cap_out = 0;
+};
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                             \
+  do {                                                                             \
+    cudaError_t e_ = (expr);                                                       \
+    if (e_ != cudaSuccess)                                                         \
+      return fail(e_ == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA,      \
+                  "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+int next_pow2_log2(int64_t x) {
+  int l = 0;
+  while ((1ll << l) < x) ++l;
+  return l;
+}
+
+// Validation (create_device): counts adjacency ids outside [-1, n) and
+// non-finite vector values.
+__global__ void validate_kernel(const float* __restrict__ v, int64_t nv,
+                                const int32_t* __restrict__ adj, int64_t na, int64_t n,
+                                unsigned long long* bad) {
+  unsigned long long local = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nv;
+       i += (int64_t)gridDim.x * blockDim.x)
+    local += !isfinite(v[i]);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < na;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t a = adj[i];
+    local += (a < -1 || a >= n);
+  }
+  if (local) atomicAdd(bad, local);
+}
+
+// Cosine: rows are L2-normalised once at index creation so the search
+// computes 1 - <q̂, x̂> with one dot product; zero rows stay zero (distance 1).
+__global__ void normalize_rows_kernel(float* data, int64_t n, int dpad) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n;
+       r += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    float* row = data + r * dpad;
+    float s = 0.f;
+    for (int i = lane; i < dpad; i += 32) s += row[i] * row[i];
+    for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    float inv = s > 0.f ? 1.0f / sqrtf(s) : 0.f;
+    for (int i = lane; i < dpad; i += 32) row[i] *= inv;
+  }
+}
+
+int alloc_index(song_index* ix, int64_t n, int32_t dim, int32_t degree, song_metric metric) {
+  CUDA_TRY(cudaGetDevice(&ix->device));
+  CUDA_TRY(cudaDeviceGetAttribute(&ix->num_sms, cudaDevAttrMultiProcessorCount, ix->device));
+  ix->n = n;
+  ix->dim = dim;
+  ix->dpad = (dim + 3) & ~3;
+  ix->degree = degree;
+  ix->metric = (int)metric;
+  CUDA_TRY(cudaMalloc(&ix->d_data, (size_t)n * ix->dpad * sizeof(float)));
+  CUDA_TRY(cudaMalloc(&ix->d_adj, (size_t)n * degree * sizeof(int32_t)));
+  CUDA_TRY(cudaMalloc(&ix->d_ticket, sizeof(unsigned)));
+  CUDA_TRY(cudaMalloc(&ix->d_status, sizeof(int)));
+  CUDA_TRY(cudaMemset(ix->d_status, 0, sizeof(int)));
+  CUDA_TRY(cudaStreamCreateWithFlags(&ix->stream, cudaStreamNonBlocking));
+  ix->last_stream = ix->stream;
+  return SONG_OK;
+}
+
+void free_index(song_index* ix) {
+  if (!ix) return;
+  cudaFree(ix->d_data);
+  cudaFree(ix->d_adj);
+  cudaFree(ix->d_ticket);
+  cudaFree(ix->d_status);
+  cudaFree(ix->d_q);
+  cudaFree(ix->d_ids);
+  cudaFree(ix->d_dists);
+  if (ix->stream) cudaStreamDestroy(ix->stream);
+  delete ix;
+}
+
+int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* adjacency,
+                      int32_t degree, song_metric metric, song_index** out) {
+  if (!out) return fail(SONG_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!vectors || !adjacency) return fail(SONG_EINVAL, "vectors/adjacency is NULL");
+  if (n < 1 || dim < 1 || degree < 1) return fail(SONG_EINVAL, "n, dim and degree must be >= 1");
+  if (n > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n must fit int32 ids");
+  if (metric < SONG_L2 || metric > SONG_COSINE) return fail(SONG_EINVAL, "unknown metric %d", (int)metric);
+  if (degree > SONG_MAX_DEGREE) return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
+  if (dim > SONG_MAX_DIM) return fail(SONG_EUNSUPPORTED, "dim %d > %d", dim, SONG_MAX_DIM);
+  return SONG_OK;
+}
+
+// per-warp shared memory of the search kernel
+struct Shape {
+  int table_log2;
+  int warp_bytes;
+};
+
+Shape search_shape(int L, bool bloom, int bloom_log2_bits) {
+  Shape s;
+  int tbytes;
+  if (bloom) {
+    s.table_log2 = bloom_log2_bits > 0 ? bloom_log2_bits : next_pow2_log2(80ll * L);
+    if (s.table_log2 < 5) s.table_log2 = 5;
+    tbytes = (1 << s.table_log2) / 8;
+  } else {
+    // live keys <= |q| + |topk| + 32 new ones <= 2L + 32; load factor <= 1/2
+    s.table_log2 = next_pow2_log2(2ll * (2 * L + 32));
+    tbytes = (1 << s.table_log2) * 4;
+  }
+  s.warp_bytes = 3 * L * 8 + 32 * 8 + 32 * 4 + tbytes;
+  s.warp_bytes = (s.warp_bytes + 15) & ~15;
+  return s;
+}
+
+template <int NCH, int METRIC, bool BLOOM>
+int launch_t(const song::SearchArgs& a, int warps, int blocks_per_sm, int num_sms,
+             cudaStream_t st) {
+  auto kern = song::song_search_kernel<NCH, METRIC, BLOOM>;
+  const size_t smem = (size_t)a.warp_smem_bytes * warps;
+  CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int fit = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&fit, kern, warps * 32, smem));
+  if (fit < 1) return fail(SONG_EUNSUPPORTED, "search kernel does not fit an SM (%zu B smem)", smem);
+  int bps = blocks_per_sm > 0 ? std::min(blocks_per_sm, fit) : fit;
+  int64_t want = (a.nq + warps - 1) / warps;
+  int64_t grid = std::min<int64_t>((int64_t)bps * num_sms, want);
+  CUDA_TRY(cudaMemsetAsync(a.ticket, 0, sizeof(unsigned), st));
+  kern<<<(unsigned)grid, warps * 32, smem, st>>>(a);
+  CUDA_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+template <int NCH>
+int launch_m(const song::SearchArgs& a, int metric, bool bloom, int warps, int bps, int sms,
+             cudaStream_t st) {
+  if (metric == SONG_L2)
+    return bloom ? launch_t<NCH, 0, true>(a, warps, bps, sms, st)
+                 : launch_t<NCH, 0, false>(a, warps, bps, sms, st);
+  if (metric == SONG_IP)
+    return bloom ? launch_t<NCH, 1, true>(a, warps, bps, sms, st)
+                 : launch_t<NCH, 1, false>(a, warps, bps, sms, st);
+  return bloom ? launch_t<NCH, 2, true>(a, warps, bps, sms, st)
+               : launch_t<NCH, 2, false>(a, warps, bps, sms, st);
+}
+
+int check_params(const song_index* ix, const song_search_params* p) {
+  if (p->K < 1) return fail(SONG_EINVAL, "K must be >= 1");
+  if (p->queue_len < p->K) return fail(SONG_EINVAL, "queue_len %d < K %d", p->queue_len, p->K);
+  if (p->queue_len > SONG_MAX_QUEUE_LEN)
+    return fail(SONG_EUNSUPPORTED, "queue_len %d > %d", p->queue_len, SONG_MAX_QUEUE_LEN);
+  if (p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM)
+    return fail(SONG_EINVAL, "unknown visited kind %d", p->visited);
+  if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
+  if (p->bloom_log2_bits < 0 || p->bloom_log2_bits > 24)
+    return fail(SONG_EUNSUPPORTED, "bloom_log2_bits %d outside [0, 24]", p->bloom_log2_bits);
+  if (p->warps_per_block < 0 || p->warps_per_block > 8)
+    return fail(SONG_EINVAL, "warps_per_block %d outside [0, 8]", p->warps_per_block);
+  if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
+  if (p->reserved != 0) return fail(SONG_EINVAL, "reserved must be 0");
+  return SONG_OK;
+}
+
+int enqueue_search(song_index* ix, const song_search_params* p, const float* q, int64_t nq,
+                   int32_t* ids, float* dists, int32_t* counters, cudaStream_t st) {
+  song::SearchArgs a;
+  a.data = ix->d_data;
+  a.adj = ix->d_adj;
+  a.queries = q;
+  a.ids_out = ids;
+  a.dists_out = dists;
+  a.counters_out = counters;
+  a.ticket = ix->d_ticket;
+  a.status = ix->d_status;
+  a.n = ix->n;
+  a.nq = nq;
+  a.dim = ix->dim;
+  a.dpad = ix->dpad;
+  a.degree = ix->degree;
+  a.K = p->K;
+  a.L = p->queue_len;
+  const bool bloom = p->visited == SONG_VISITED_BLOOM;
+  Shape sh = search_shape(p->queue_len, bloom, p->bloom_log2_bits);
+  a.table_log2 = sh.table_log2;
+  a.warp_smem_bytes = sh.warp_bytes;
+  a.entry = p->entry;
+  a.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);
+  a.id_offset = p->id_offset;
+  int warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
+  while (warps > 1 && (size_t)sh.warp_bytes * warps > 200 * 1024) warps >>= 1;
+  if ((size_t)sh.warp_bytes * warps > 227 * 1024)
+    return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
+                p->queue_len, sh.warp_bytes);
+  ix->last_stream = st;
+  const int nch = (ix->dpad + 127) / 128;
+  if (nch <= 1) return launch_m<1>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
+  if (nch <= 2) return launch_m<2>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
+  if (nch <= 4) return launch_m<4>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
+  return launch_m<8>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
+}
+
+int finish_create(song_index* ix, cudaStream_t st) {
+  if (ix->metric == SONG_COSINE) {
+    int blocks = (int)std::min<int64_t>((ix->n + 7) / 8, 65535);
+    normalize_rows_kernel<<<blocks, 256, 0, st>>>(ix->d_data, ix->n, ix->dpad);
+    CUDA_TRY(cudaGetLastError());
+  }
+  CUDA_TRY(cudaStreamSynchronize(st));
+  return SONG_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void song_default_params(song_search_params* p, int32_t K, int32_t queue_len) {
+  if (!p) return;
+  std::memset(p, 0, sizeof *p);
+  p->K = K;
+  p->queue_len = queue_len;
+  p->visited = SONG_VISITED_HASH;
+}
+
+int song_index_create(const float* vectors, int64_t n, int32_t dim, const int32_t* adjacency,
+                      int32_t degree, song_metric metric, song_index** out) {
+  int rc = check_create_args(vectors, n, dim, adjacency, degree, metric, out);
+  if (rc) return rc;
+  for (int64_t i = 0; i < n * (int64_t)degree; ++i)
+    if (adjacency[i] < -1 || adjacency[i] >= n)
+      return fail(SONG_EINVAL, "adjacency[%lld] = %d outside [-1, %lld)", (long long)i,
+                  adjacency[i], (long long)n);
+  for (int64_t i = 0; i < n * (int64_t)dim; ++i)
+    if (!std::isfinite(vectors[i]))
+      return fail(SONG_EINVAL, "vectors[%lld] is not finite", (long long)i);
+  song_index* ix = new song_index();
+  rc = alloc_index(ix, n, dim, degree, metric);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  cudaError_t e = cudaMemsetAsync(ix->d_data, 0, (size_t)n * ix->dpad * sizeof(float), ix->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpy2DAsync(ix->d_data, ix->dpad * sizeof(float), vectors, dim * sizeof(float),
+                          dim * sizeof(float), n, cudaMemcpyHostToDevice, ix->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(ix->d_adj, adjacency, (size_t)n * degree * sizeof(int32_t),
+                        cudaMemcpyHostToDevice, ix->stream);
+  if (e != cudaSuccess) {
+    free_index(ix);
+    return fail(SONG_ECUDA, "index upload: %s", cudaGetErrorString(e));
+  }
+  rc = finish_create(ix, ix->stream);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  *out = ix;
+  return SONG_OK;
+}
+
+int song_index_create_device(const float* vectors, int64_t n, int32_t dim,
+                             const int32_t* adjacency, int32_t degree, song_metric metric,
+                             void* stream, song_index** out) {
+  int rc = check_create_args(vectors, n, dim, adjacency, degree, metric, out);
+  if (rc) return rc;
+  cudaStream_t st = (cudaStream_t)stream;
+  unsigned long long* d_bad = nullptr;
+  CUDA_TRY(cudaMalloc(&d_bad, sizeof *d_bad));
+  CUDA_TRY(cudaMemsetAsync(d_bad, 0, sizeof *d_bad, st));
+  validate_kernel<<<1184, 256, 0, st>>>(vectors, n * (int64_t)dim, adjacency, n * (int64_t)degree,
+                                        n, d_bad);
+  unsigned long long bad = 0;
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&bad, d_bad, sizeof bad, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  cudaFree(d_bad);
+  if (e != cudaSuccess) return fail(SONG_ECUDA, "validation: %s", cudaGetErrorString(e));
+  if (bad) return fail(SONG_EINVAL, "%llu invalid adjacency ids / non-finite values", bad);
+  song_index* ix = new song_index();
+  rc = alloc_index(ix, n, dim, degree, metric);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  e = cudaMemsetAsync(ix->d_data, 0, (size_t)n * ix->dpad * sizeof(float), st);
+  if (e == cudaSuccess)
+    e = cudaMemcpy2DAsync(ix->d_data, ix->dpad * sizeof(float), vectors, dim * sizeof(float),
+                          dim * sizeof(float), n, cudaMemcpyDeviceToDevice, st);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(ix->d_adj, adjacency, (size_t)n * degree * sizeof(int32_t),
+                        cudaMemcpyDeviceToDevice, st);
+  if (e != cudaSuccess) {
+    free_index(ix);
+    return fail(SONG_ECUDA, "index copy: %s", cudaGetErrorString(e));
+  }
+  rc = finish_create(ix, st);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  *out = ix;
+  return SONG_OK;
+}
+
+int song_index_destroy(song_index* idx) {
+  if (!idx) return SONG_OK;
+  cudaStreamSynchronize(idx->last_stream);
+  free_index(idx);
+  return SONG_OK;
+}
+
+int song_index_get_info(const song_index* ix, song_index_info* info) {
+  if (!ix || !info) return fail(SONG_EINVAL, "NULL argument");
+  info->n = ix->n;
+  info->dim = ix->dim;
+  info->dim_padded = ix->dpad;
+  info->degree = ix->degree;
+  info->metric = ix->metric;
+  info->vector_bytes = ix->n * (int64_t)ix->dpad * 4;
+  info->graph_bytes = ix->n * (int64_t)ix->degree * 4;
+  info->device = ix->device;
+  info->num_sms = ix->num_sms;
+  return SONG_OK;
+}
+
+int song_search_ex(song_index* ix, const song_search_params* p, const float* queries, int64_t nq,
+                   int32_t* ids_out, float* dists_out, int32_t* counters_out, void* stream) {
+  if (!ix || !p || !queries || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (nq < 1) return fail(SONG_EINVAL, "nq must be >= 1");
+  if (nq > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "nq must fit int32");
+  int rc = check_params(ix, p);
+  if (rc) return rc;
+  return enqueue_search(ix, p, queries, nq, ids_out, dists_out, counters_out,
+                        (cudaStream_t)stream);
+}
+
+int song_index_last_status(song_index* ix) {
+  if (!ix) return fail(SONG_EINVAL, "NULL index");
+  CUDA_TRY(cudaStreamSynchronize(ix->last_stream));
+  int st = 0;
+  CUDA_TRY(cudaMemcpy(&st, ix->d_status, sizeof st, cudaMemcpyDeviceToHost));
+  CUDA_TRY(cudaMemset(ix->d_status, 0, sizeof st));
+  if (st & song::STATUS_BAD_INPUT) return fail(SONG_EINVAL, "a query had a non-finite value");
+  if (st & song::STATUS_ITER_CAP) return fail(SONG_EITERCAP, "a query reached max_iters");
+  return SONG_OK;
+}
+
+int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int32_t queue_len,
+                int32_t* ids_out, float* dists_out) {
+  if (!ix || !queries || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (nq < 1) return fail(SONG_EINVAL, "nq must be >= 1");
+  song_search_params p;
+  song_default_params(&p, K, queue_len);
+  int rc = check_params(ix, &p);
+  if (rc) return rc;
+  const size_t qbytes = (size_t)nq * ix->dim * sizeof(float);
+  const size_t obytes = (size_t)nq * K * sizeof(int32_t);
+  if (qbytes > ix->cap_q) {
+    cudaFree(ix->d_q);
+    ix->d_q = nullptr;
+    ix->cap_q = 0;
+    CUDA_TRY(cudaMalloc(&ix->d_q, qbytes));
+    ix->cap_q = qbytes;
+  }
+  if (obytes > ix->cap_out) {
+    cudaFree(ix->d_ids);
+    cudaFree(ix->d_dists);
+    ix->d_ids = nullptr;
+    ix->d_dists = nullptr;
+    ix->cap_out = 0;
+    CUDA_TRY(cudaMalloc(&ix->d_ids, obytes));
+    CUDA_TRY(cudaMalloc(&ix->d_dists, obytes));
+    ix->cap_out = obytes;
+  }
+  cudaStream_t st = ix->stream;
+  CUDA_TRY(cudaMemcpyAsync(ix->d_q, queries, qbytes, cudaMemcpyHostToDevice, st));
+  rc = enqueue_search(ix, &p, ix->d_q, nq, ix->d_ids, ix->d_dists, nullptr, st);
+  if (rc) return rc;
+  CUDA_TRY(cudaMemcpyAsync(ids_out, ix->d_ids, obytes, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaMemcpyAsync(dists_out, ix->d_dists, obytes, cudaMemcpyDeviceToHost, st));
+  return song_index_last_status(ix);
+}
+
+int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,
+                    int32_t Kin, int32_t K, int32_t* ids_out, float* dists_out, void* stream) {
+  if (!ids_in || !dists_in || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (G < 1 || nq < 1 || Kin < 1 || K < 1) return fail(SONG_EINVAL, "sizes must be >= 1");
+  if (K > 1024 || Kin > 1024) return fail(SONG_EUNSUPPORTED, "K and Kin must be <= 1024");
+  const int warps = 8;
+  int64_t blocks = (nq + warps - 1) / warps;
+  song::song_merge_kernel<<<(unsigned)blocks, warps * 32, 0, (cudaStream_t)stream>>>(
+      ids_in, dists_in, G, nq, Kin, K, ids_out, dists_out);
+  CUDA_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+const char* song_last_error(void) { return g_err.c_str(); }
+
+const char* song_version(void) { return "song-b200 0.1 sm_100a"; }
+
+}  // extern "C"

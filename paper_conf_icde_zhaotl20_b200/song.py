@@ -1,0 +1,250 @@
+"""Thin Python binding of libsong.so (include/song.h): argument marshalling only.
+
+Every step of the search runs in the sm_100a kernels behind the C ABI; this
+module never computes a distance, a queue or a visited set, and there is no
+CPU fallback: if libsong.so or a CUDA device is missing, calls raise.
+
+torch is used only for device memory and streams: CUDA tensors are passed to
+``song_search_ex`` as raw device pointers on torch's current stream.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Optional, Tuple
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libsong.so")
+
+L2, IP, COSINE = 0, 1, 2
+METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
+VISITED_HASH, VISITED_BLOOM = 0, 1
+VISITED = {"hash": VISITED_HASH, "bloom": VISITED_BLOOM}
+
+STATUS = {0: "SONG_OK", -1: "SONG_EINVAL", -2: "SONG_ENOMEM", -3: "SONG_ECUDA",
+          -4: "SONG_EUNSUPPORTED", -5: "SONG_EITERCAP"}
+
+EXPORTED = ["song_default_params", "song_index_create", "song_index_create_device",
+            "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
+            "song_index_last_status", "song_merge_topk", "song_last_error", "song_version"]
+
+
+class SongError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+class SearchParams(ctypes.Structure):
+    _fields_ = [("K", ctypes.c_int32), ("queue_len", ctypes.c_int32),
+                ("visited", ctypes.c_int32), ("bloom_log2_bits", ctypes.c_int32),
+                ("entry", ctypes.c_int32), ("max_iters", ctypes.c_int32),
+                ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
+                ("id_offset", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+
+
+class IndexInfo(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("dim", ctypes.c_int32), ("dim_padded", ctypes.c_int32),
+                ("degree", ctypes.c_int32), ("metric", ctypes.c_int32),
+                ("vector_bytes", ctypes.c_int64), ("graph_bytes", ctypes.c_int64),
+                ("device", ctypes.c_int32), ("num_sms", ctypes.c_int32)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libsong.so (raises if it was not built: no fallback exists)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                              "(there is no CPU fallback for the SONG search)")
+        L = ctypes.CDLL(LIB_PATH)
+        P, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        PP = ctypes.POINTER(ctypes.c_void_p)
+        L.song_default_params.restype = None
+        L.song_default_params.argtypes = [ctypes.POINTER(SearchParams), i32, i32]
+        L.song_index_create.argtypes = [P, i64, i32, P, i32, i32, PP]
+        L.song_index_create_device.argtypes = [P, i64, i32, P, i32, i32, P, PP]
+        L.song_index_destroy.argtypes = [P]
+        L.song_index_get_info.argtypes = [P, ctypes.POINTER(IndexInfo)]
+        L.song_search.argtypes = [P, P, i64, i32, i32, P, P]
+        L.song_search_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
+        L.song_index_last_status.argtypes = [P]
+        L.song_merge_topk.argtypes = [P, P, i32, i64, i32, i32, P, P, P]
+        L.song_last_error.restype = ctypes.c_char_p
+        L.song_last_error.argtypes = []
+        L.song_version.restype = ctypes.c_char_p
+        L.song_version.argtypes = []
+        for name in ("song_index_create", "song_index_create_device", "song_index_destroy",
+                     "song_index_get_info", "song_search", "song_search_ex",
+                     "song_index_last_status", "song_merge_topk"):
+            getattr(L, name).restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise SongError(rc, lib().song_last_error().decode())
+
+
+def _torch():
+    import torch  # plumbing only: device memory + streams
+    return torch
+
+
+def _is_cuda_tensor(x) -> bool:
+    try:
+        torch = _torch()
+    except ImportError:
+        return False
+    return isinstance(x, torch.Tensor) and x.is_cuda
+
+
+def _stream_ptr(device) -> ctypes.c_void_p:
+    torch = _torch()
+    return ctypes.c_void_p(torch.cuda.current_stream(device).cuda_stream)
+
+
+@dataclass
+class Params:
+    """song_search_params (include/song.h)."""
+    K: int = 10
+    queue_len: int = 64
+    visited: str = "hash"
+    bloom_log2_bits: int = 0
+    entry: int = 0
+    max_iters: int = 0
+    warps_per_block: int = 0
+    blocks_per_sm: int = 0
+    id_offset: int = 0
+
+    def to_c(self) -> SearchParams:
+        p = SearchParams()
+        lib().song_default_params(ctypes.byref(p), self.K, self.queue_len)
+        p.visited = VISITED[self.visited]
+        p.bloom_log2_bits = self.bloom_log2_bits
+        p.entry = self.entry
+        p.max_iters = self.max_iters
+        p.warps_per_block = self.warps_per_block
+        p.blocks_per_sm = self.blocks_per_sm
+        p.id_offset = self.id_offset
+        return p
+
+
+class SongIndex:
+    """song_index_create / song_search / song_index_destroy.
+
+    ``vectors`` [n, dim] float32 and ``adjacency`` [n, degree] int32 may be
+    numpy arrays (host create) or CUDA tensors (device create)."""
+
+    def __init__(self, vectors, adjacency, metric: str = "l2"):
+        self._h = ctypes.c_void_p()
+        self.metric = metric
+        m = METRICS[metric]
+        if _is_cuda_tensor(vectors):
+            torch = _torch()
+            v = vectors.contiguous().to(torch.float32)
+            a = adjacency.to(device=v.device, dtype=torch.int32).contiguous()
+            self.device = v.device
+            with torch.cuda.device(v.device):
+                _check(lib().song_index_create_device(
+                    ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1],
+                    ctypes.c_void_p(a.data_ptr()), a.shape[1], m, _stream_ptr(v.device),
+                    ctypes.byref(self._h)))
+        else:
+            v = np.ascontiguousarray(vectors, np.float32)
+            a = np.ascontiguousarray(adjacency, np.int32)
+            assert v.ndim == 2 and a.ndim == 2 and a.shape[0] == v.shape[0]
+            self.device = None
+            _check(lib().song_index_create(
+                v.ctypes.data_as(ctypes.c_void_p), v.shape[0], v.shape[1],
+                a.ctypes.data_as(ctypes.c_void_p), a.shape[1], m, ctypes.byref(self._h)))
+        info = self.info()
+        self.n, self.dim, self.degree = info.n, info.dim, info.degree
+
+    def info(self) -> IndexInfo:
+        inf = IndexInfo()
+        _check(lib().song_index_get_info(self._h, ctypes.byref(inf)))
+        return inf
+
+    def search_host(self, queries: np.ndarray, K: int, queue_len: int) -> Tuple[np.ndarray, np.ndarray]:
+        """song_search: HOST buffers in and out (HtoD + kernel + DtoH inside)."""
+        q = np.ascontiguousarray(queries, np.float32)
+        if q.ndim == 1:
+            q = q[None]
+        ids = np.empty((q.shape[0], K), np.int32)
+        dists = np.empty((q.shape[0], K), np.float32)
+        self.search_host_into(q, K, queue_len, ids, dists)
+        return ids, dists
+
+    def search_host_into(self, q, K, queue_len, ids, dists):
+        """song_search into caller buffers (numpy or pinned CPU tensors)."""
+        def ptr(x):
+            return ctypes.c_void_p(x.data_ptr() if hasattr(x, "data_ptr") else
+                                   x.ctypes.data)
+        _check(lib().song_search(self._h, ptr(q), q.shape[0], K, queue_len, ptr(ids), ptr(dists)))
+
+    def search(self, queries, K: int = 10, queue_len: int = 64, params: Optional[Params] = None,
+               counters: bool = False, out=None):
+        """song_search_ex on CUDA tensors (async on torch's current stream).
+        Returns (ids [nq,K] int32, dists [nq,K] f32[, counters [nq,2] int32])."""
+        torch = _torch()
+        if not _is_cuda_tensor(queries):
+            raise TypeError("search() takes a CUDA tensor; use search_host() for host arrays")
+        p = params or Params(K=K, queue_len=queue_len)
+        q = queries.contiguous()
+        if q.dtype != torch.float32:
+            q = q.float()
+        nq = q.shape[0]
+        if out is None:
+            ids = torch.empty((nq, p.K), dtype=torch.int32, device=q.device)
+            dists = torch.empty((nq, p.K), dtype=torch.float32, device=q.device)
+            ctr = torch.empty((nq, 2), dtype=torch.int32, device=q.device) if counters else None
+        else:
+            ids, dists, ctr = out
+        cp = p.to_c()
+        _check(lib().song_search_ex(
+            self._h, ctypes.byref(cp), ctypes.c_void_p(q.data_ptr()), nq,
+            ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(dists.data_ptr()),
+            ctypes.c_void_p(ctr.data_ptr() if ctr is not None else 0), _stream_ptr(q.device)))
+        return (ids, dists, ctr) if counters else (ids, dists)
+
+    def last_status(self):
+        """Synchronise and raise SongError if a query was flagged."""
+        _check(lib().song_index_last_status(self._h))
+
+    def close(self):
+        if self._h:
+            lib().song_index_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def merge_topk(ids, dists, K: int):
+    """song_merge_topk: ids/dists [G, nq, Kin] CUDA tensors (rows sorted by
+    (dist, id), global ids) -> the K best per query [nq, K]."""
+    torch = _torch()
+    ids = ids.to(torch.int32).contiguous()
+    dists = dists.to(torch.float32).contiguous()
+    G, nq, kin = ids.shape
+    oi = torch.empty((nq, K), dtype=torch.int32, device=ids.device)
+    od = torch.empty((nq, K), dtype=torch.float32, device=ids.device)
+    _check(lib().song_merge_topk(ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(dists.data_ptr()),
+                                 G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
+                                 ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
+    return oi, od
+
+
+def version() -> str:
+    return lib().song_version().decode()

@@ -1,0 +1,262 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+Bars (BASELINE.json north_star):
+ * integer-valued data (pin P8): ids, distances AND counters bit-exact for
+   every query;
+ * float data: top-K ids identical on >= 99.5 % of queries, distances within
+   rtol 1e-5 + atol 1e-5 * scale, recall within 0.002 of the oracle's.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from workloads.graph import build_graph  # noqa: E402
+from workloads.synth import CONFIGS, make_data  # noqa: E402
+
+from _golden import golden_path  # noqa: E402
+import test_oracle_pins as pins  # noqa: E402
+
+
+def song():
+    from paper_conf_icde_zhaotl20_b200 import song as s
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return s
+
+
+ORACLE_FLAGS = {"hash": oracle.OPTIMIZED, "bloom": oracle.OPTIMIZED_BLOOM}
+
+
+def gpu_search(idx, q, K, L, visited="hash", **kw):
+    s = song()
+    p = s.Params(K=K, queue_len=L, visited=visited, **kw)
+    qt = torch.as_tensor(q, device="cuda")
+    ids, d, c = idx.search(qt, params=p, counters=True)
+    torch.cuda.synchronize()
+    idx.last_status()
+    return ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy()
+
+
+def bloom_bits_for(L, log2=0):
+    return (1 << log2) if log2 else oracle.default_bloom_bits(L)
+
+
+def assert_exact(g, o):
+    gi, gd, gc = g
+    oi, od, oc = o[:3]
+    np.testing.assert_array_equal(gi, oi)
+    np.testing.assert_array_equal(gd, od)
+    np.testing.assert_array_equal(gc.astype(np.int64), oc)
+
+
+def assert_close(g, o, truth=None, id_frac=0.995, scale=1.0):
+    gi, gd, _ = g
+    oi, od = o[0], o[1]
+    same = (gi == oi).all(1).mean()
+    assert same >= id_frac, f"only {same:.4f} of queries have identical top-K ids"
+    ok = gi == oi
+    np.testing.assert_allclose(gd[ok], od[ok], rtol=1e-5, atol=1e-5 * scale)
+    if truth is not None:
+        assert abs(oracle.recall(gi, truth) - oracle.recall(oi, truth)) <= 0.002
+
+
+# ---------------------------------------------------------------- toy / P1-P2
+@pytest.mark.parametrize("visited", ["hash", "bloom"])
+def test_fig1_toy_on_gpu(visited):
+    data, adj, _, result = pins.load_toy()
+    s = song()
+    idx = s.SongIndex(data, adj)
+    ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited)
+    assert [int(x) + 1 for x in ids[0]] == result
+    if visited == "hash":
+        assert c[0].tolist() == [12, 4]  # Fig. 4(c): 12 distances, 4 expansions
+    o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
+                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(3))
+    assert_exact((ids, d, c), o)
+
+
+# ----------------------------------------------------------------- tiny config
+@pytest.fixture(scope="module")
+def tiny():
+    cfg = CONFIGS["tiny"]
+    x, q = make_data(cfg)
+    adj = build_graph(x, degree=cfg.degree, row_block=2048, col_block=16384).numpy()
+    xn, qn = x.numpy(), q.numpy()
+    truth, _ = oracle.bruteforce(xn, qn, cfg.K, nthreads=8)
+    return cfg, xn, qn, adj, truth
+
+
+@pytest.mark.parametrize("L", [10, 64, 257])
+@pytest.mark.parametrize("visited", ["hash", "bloom"])
+def test_tiny_parity(tiny, L, visited):
+    cfg, x, q, adj, truth = tiny
+    s = song()
+    idx = s.SongIndex(x, adj)
+    g = gpu_search(idx, q, cfg.K, L, visited)
+    o = oracle.search(x, adj, q, cfg.K, L, flags=ORACLE_FLAGS[visited],
+                      bloom_bits=bloom_bits_for(L))
+    assert_close(g, o, truth, scale=float(np.abs(o[1]).max()))
+
+
+# -------------------------------------------- integer data: bit-exact (P8)
+@pytest.fixture(scope="module")
+def sift100k():
+    cfg = CONFIGS["sift1m"]
+    x, q = make_data(cfg, device="cuda", n=100_000, nq=500)
+    adj = build_graph(x, degree=32)
+    return cfg, x, q, adj
+
+
+@pytest.mark.parametrize("L,visited,warps", [(10, "hash", 4), (16, "hash", 1), (64, "hash", 4),
+                                            (200, "hash", 8), (64, "bloom", 4),
+                                            (1024, "hash", 2)])
+def test_sift_integer_bit_exact(sift100k, L, visited, warps):
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    g = gpu_search(idx, q.cpu().numpy(), cfg.K, L, visited, warps_per_block=warps)
+    o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, L,
+                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L), nthreads=8)
+    assert_exact(g, o)
+
+
+def test_sift_small_bloom_filter_exact(sift100k):
+    """A deliberately small Bloom filter (2^9 bits) saturates: false positives
+    change the search, and the GPU must follow the oracle's spec bit by bit."""
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    g = gpu_search(idx, q.cpu().numpy(), cfg.K, 48, "bloom", bloom_log2_bits=9)
+    o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, 48,
+                      flags=oracle.OPTIMIZED_BLOOM, bloom_bits=1 << 9, nthreads=8)
+    assert_exact(g, o)
+
+
+def test_host_and_device_entry_points_agree(sift100k):
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)  # device create
+    idx2 = s.SongIndex(x.cpu().numpy(), adj.cpu().numpy())  # host create
+    qi, qd = idx2.search_host(q.cpu().numpy(), cfg.K, 64)
+    g = gpu_search(idx, q.cpu().numpy(), cfg.K, 64)
+    np.testing.assert_array_equal(qi, g[0])
+    np.testing.assert_array_equal(qd, g[1])
+
+
+# ------------------------------------------------ other metrics / dimensions
+@pytest.mark.parametrize("name,n", [("glove200", 30_000), ("nytimes256", 30_000),
+                                    ("gist1m", 20_000)])
+def test_metric_and_dim_parity(name, n):
+    cfg = CONFIGS[name]
+    x, q = make_data(cfg, device="cuda", n=n, nq=200)
+    adj = build_graph(x, degree=cfg.degree, metric=cfg.metric)
+    s = song()
+    idx = s.SongIndex(x, adj, metric=cfg.metric)
+    xn, qn, an = x.cpu().numpy(), q.cpu().numpy(), adj.cpu().numpy()
+    m = oracle.METRICS[cfg.metric]
+    truth, _ = oracle.bruteforce(xn, qn, cfg.K, metric=m, nthreads=8)
+    for L in (32, 128):
+        g = gpu_search(idx, qn, cfg.K, L)
+        o = oracle.search(xn, an, qn, cfg.K, L, metric=m, nthreads=8)
+        assert_close(g, o, truth, id_frac=0.99 if name == "nytimes256" else 0.995,
+                     scale=float(np.abs(o[1]).max()))
+
+
+# ------------------------------------------------------------------- edges
+def small_random(n=3000, dim=30, deg=12, seed=0, integer=True):
+    rng = np.random.default_rng(seed)
+    x = rng.integers(0, 20, (n, dim)).astype(np.float32) if integer else \
+        rng.standard_normal((n, dim)).astype(np.float32)
+    adj = rng.integers(-1, n, (n, deg)).astype(np.int32)
+    adj[:, 0] = (np.arange(n) + 1) % n
+    adj[:, 3] = adj[:, 2]  # repeated ids inside a row
+    q = rng.integers(0, 20, (64, dim)).astype(np.float32) if integer else \
+        rng.standard_normal((64, dim)).astype(np.float32)
+    return x, adj, q
+
+
+@pytest.mark.parametrize("dim", [1, 3, 30, 130, 257])
+@pytest.mark.parametrize("L,K", [(1, 1), (7, 7), (33, 10), (100, 100)])
+def test_edges_exact(dim, L, K):
+    """ragged dims (row padding), degree < 32 with -1 padding and repeats,
+    L = K = 1 (greedy), K = L, queue sizes that are not multiples of 32."""
+    x, adj, q = small_random(dim=dim)
+    s = song()
+    idx = s.SongIndex(x, adj)
+    for visited in ("hash", "bloom"):
+        g = gpu_search(idx, q, K, L, visited)
+        o = oracle.search(x, adj, q, K, L, flags=ORACLE_FLAGS[visited],
+                          bloom_bits=bloom_bits_for(L))
+        assert_exact(g, o)
+
+
+def test_entry_offset_and_unreachable_padding():
+    x, adj, q = small_random(n=500, dim=8)
+    adj2 = adj.copy()
+    adj2[:] = -1
+    adj2[5, :3] = [6, 7, 8]  # only 4 vertices reachable from entry 5
+    s = song()
+    idx = s.SongIndex(x, adj2)
+    g = gpu_search(idx, q, 10, 16, entry=5, id_offset=1000)
+    assert (g[0][:, :4] >= 1000).all() and (g[0][:, 4:] == -1).all()
+    assert np.isinf(g[1][:, 4:]).all()
+    o = oracle.search(x, adj2, q, 10, 16, entry=5)
+    np.testing.assert_array_equal(np.where(g[0] >= 0, g[0] - 1000, -1), o[0])
+
+
+def test_large_queue_len_max():
+    x, adj, q = small_random(n=5000, dim=16, deg=32)
+    s = song()
+    idx = s.SongIndex(x, adj)
+    g = gpu_search(idx, q[:16], 100, 2048)
+    o = oracle.search(x, adj, q[:16], 100, 2048)
+    assert_exact(g, o)
+
+
+def test_errors():
+    s = song()
+    x, adj, q = small_random(n=100, dim=4)
+    bad = adj.copy()
+    bad[3, 1] = 100
+    with pytest.raises(s.SongError, match="EINVAL"):
+        s.SongIndex(x, bad)
+    with pytest.raises(s.SongError, match="EINVAL"):
+        s.SongIndex(torch.as_tensor(x, device="cuda"), torch.as_tensor(bad, device="cuda"))
+    xn = x.copy()
+    xn[2, 2] = np.nan
+    with pytest.raises(s.SongError, match="EINVAL"):
+        s.SongIndex(xn, adj)
+    idx = s.SongIndex(x, adj)
+    with pytest.raises(s.SongError, match="EINVAL"):
+        idx.search_host(q, 10, 5)  # queue_len < K
+    with pytest.raises(s.SongError, match="EUNSUPPORTED"):
+        idx.search_host(q, 10, 4096)
+    qb = q.copy()
+    qb[1, 0] = np.inf
+    with pytest.raises(s.SongError, match="EINVAL"):
+        idx.search_host(qb, 10, 16)
+    with pytest.raises(s.SongError, match="EITERCAP"):
+        gpu_search(idx, q, 10, 64, max_iters=2)
+
+
+# ----------------------------------------------------------------- merge
+def test_merge_topk_matches_plain_merge():
+    rng = np.random.default_rng(0)
+    G, nq, kin, K = 4, 300, 20, 10
+    ids = np.full((G, nq, kin), -1, np.int32)
+    dists = np.full((G, nq, kin), np.inf, np.float32)
+    for g in range(G):
+        for r in range(nq):
+            m = rng.integers(0, kin + 1)
+            d = np.sort(rng.integers(0, 50, m).astype(np.float32))
+            i = rng.choice(1000, m, replace=False) + g * 1000
+            order = np.lexsort((i, d))
+            ids[g, r, :m] = i[order]
+            dists[g, r, :m] = d[order]
+    s = song()
+    oi, od = s.merge_topk(torch.as_tensor(ids, device="cuda"), torch.as_tensor(dists, device="cuda"), K)
+    ei, ed = oracle.merge_shards(list(ids), list(dists), K)
+    np.testing.assert_array_equal(oi.cpu().numpy(), ei)
+    np.testing.assert_array_equal(od.cpu().numpy(), ed)
