@@ -5,19 +5,25 @@
 // of Algorithm 1 runs the paper's three stages (§III, Fig. 3)
 // warp-cooperatively instead of on "one single thread":
 //
-//   maintain/pop  q head is read by all lanes; topk insertion is a warp ballot
-//                 rank + in-place shift (§IV-C bounded topk, reading A1)
-//   locate (§V)   lane j loads adjacency slot j (one coalesced 128 B row),
-//                 drops padding, repeats (match.any) and visited ids (parallel
-//                 hash probes) and compacts survivors with a ballot
-//   distance (§VI) LDG.128 gathers of R candidate rows per batch, every lane a
-//                 16 B slice of each row; a transposed butterfly reduces R
-//                 partial sums in R-1+(5-log2 R) shuffles (P:455's shfl_down
-//                 reduction, batched)
-//   maintain      selected insertion (§IV-D) against topk's max, warp bitonic
-//                 sort of the <= 32 survivors, visited insert, merge-path merge
-//                 into the bounded q (§IV-C) with visited deletion of the
-//                 evicted keys (§IV-E)
+//   locate (§V)    the adjacency row of the head (prefetched into registers
+//                  during the previous iteration's maintenance) is filtered:
+//                  padding, repeats (match.any, only if the index has them)
+//                  and visited ids (32 parallel hash probes), compacted by a
+//                  ballot
+//   distance (§VI) every surviving candidate lane issues ONE bulk copy
+//                  (cp.async.bulk, the TMA engine) of its d*4-byte row into a
+//                  per-warp shared-memory stage, completion on an mbarrier:
+//                  all rows of the iteration are in flight at once with no
+//                  register cost.  Lanes then read 16 B slices (LDS.128,
+//                  conflict-free) and a transposed butterfly reduces R rows in
+//                  R-1+(5-log2 R) shuffles (P:455's shfl_down reduction,
+//                  batched)
+//   maintain (§IV) selected insertion (§IV-D) against topk's max, warp bitonic
+//                  sort of the <= 32 survivors, visited insert, bitonic merge
+//                  into the bounded q (§IV-C) with visited deletion of the
+//                  evicted keys (§IV-E).  For queue_len <= 128 q and topk live
+//                  in registers (sorted, striped over the lanes); larger
+//                  queues use shared-memory arrays and merge-path ranks.
 //
 // Priority-queue keys are u64 (orderable(dist) << 32 | id): the (dist, id)
 // total order of DESIGN.md reading A3 as a single integer compare.
@@ -32,27 +38,32 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int EMPTY = -1;  // hash slot never used
 constexpr int TOMB = -2;   // hash slot whose key was deleted (§IV-E)
 constexpr uint64_t KEY_MAX = ~0ull;
+constexpr int STAGE_BYTES = 16384;  // per-warp row stage (32 rows of d = 128)
 
 enum : int { STATUS_BAD_INPUT = 1, STATUS_ITER_CAP = 2 };
+enum : int { MET_L2 = 0, MET_DOT = 1 };
 
 struct SearchArgs {
-  const float* data;   // [n][dpad], 16 B aligned rows
-  const int32_t* adj;  // [n][degree]
-  const float* queries;  // [nq][dim] (caller layout, unpadded)
-  int32_t* ids_out;      // [nq][K]
-  float* dists_out;      // [nq][K]
-  int32_t* counters_out; // [nq][2] or nullptr
-  unsigned* ticket;      // work counter, zeroed before launch
-  int* status;           // sticky STATUS_* bits
+  const float* data;      // [n][dpad], 16 B aligned rows
+  const int32_t* adj;     // [n][degree]
+  const float* queries;   // [nq][dim] (caller layout, unpadded)
+  int32_t* ids_out;       // [nq][K]
+  float* dists_out;       // [nq][K]
+  int32_t* counters_out;  // [nq][2] or nullptr
+  unsigned* ticket;       // work counter, zeroed before launch
+  int* status;            // sticky STATUS_* bits
   int64_t n;
   int64_t nq;
   int dim, dpad, degree;
   int K, L;
   int table_log2;  // hash: log2 slots; bloom: log2 bits
   int entry, max_iters, id_offset;
+  int cosine;      // MET_DOT: 1 -> 1 - dot, 0 -> -dot
+  int dedup;       // 1 if some adjacency row repeats an id
   int warp_smem_bytes;
 };
 
+// ------------------------------------------------------------------- keys --
 __device__ __forceinline__ uint32_t f2ord(float f) {
   f = f + 0.0f;  // canonicalise -0.0 to +0.0 (reading A9)
   uint32_t u = __float_as_uint(f);
@@ -76,12 +87,55 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   return m;
 }
 
-__device__ __forceinline__ float4 ldg_f4(const float4* p) {
-  float4 r;
-  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
-               : "l"(p));
-  return r;
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a < b ? b : a; }
+
+// warp-wide minimum of a u64 key (two REDUX ops)
+__device__ __forceinline__ uint64_t warp_min_key(uint64_t k) {
+  uint32_t hi = (uint32_t)(k >> 32);
+  uint32_t mh = __reduce_min_sync(FULL, hi);
+  uint32_t lo = (hi == mh) ? (uint32_t)k : 0xffffffffu;
+  uint32_t ml = __reduce_min_sync(FULL, lo);
+  return ((uint64_t)mh << 32) | ml;
+}
+
+// ------------------------------------------------------- async row copies --
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+// one bulk copy (TMA engine) of `bytes` from global to shared, completing on bar
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
 // ---------------------------------------------------------------- visited --
@@ -145,7 +199,7 @@ struct BloomSet {
   int log2;  // m = 2^log2 bits
   __device__ __forceinline__ bool contains(int v) const {
     uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
-    uint32_t mask = (log2 >= 32) ? 0xffffffffu : ((1u << log2) - 1);
+    uint32_t mask = (1u << log2) - 1;
 #pragma unroll
     for (int i = 0; i < 7; ++i) {
       uint32_t b = (h1 + (uint32_t)i * h2) & mask;
@@ -155,7 +209,7 @@ struct BloomSet {
   }
   __device__ __forceinline__ void insert(int v) {
     uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
-    uint32_t mask = (log2 >= 32) ? 0xffffffffu : ((1u << log2) - 1);
+    uint32_t mask = (1u << log2) - 1;
 #pragma unroll
     for (int i = 0; i < 7; ++i) {
       uint32_t b = (h1 + (uint32_t)i * h2) & mask;
@@ -165,17 +219,16 @@ struct BloomSet {
 };
 
 // ------------------------------------------------------------- utilities --
+template <bool DESC>
 __device__ __forceinline__ uint64_t bitonic_sort32(uint64_t key, int lane) {
 #pragma unroll
   for (int k = 2; k <= 32; k <<= 1) {
 #pragma unroll
     for (int j = k >> 1; j > 0; j >>= 1) {
       uint64_t other = __shfl_xor_sync(FULL, key, j);
-      bool ascending = (lane & k) == 0;
+      bool ascending = ((lane & k) == 0) != DESC;
       bool lower = (lane & j) == 0;
-      uint64_t lo = key < other ? key : other;
-      uint64_t hi = key < other ? other : key;
-      key = (lower == ascending) ? lo : hi;
+      key = (lower == ascending) ? umin64(key, other) : umax64(key, other);
     }
   }
   return key;
@@ -226,52 +279,149 @@ __device__ __forceinline__ float transpose_reduce(float (&v)[R], int lane) {
   return r;
 }
 
+// --------------------------------------------------- register queues (<=128)
+// QR u64 registers per lane hold a sorted array of 32*QR keys: element
+// e = r*32 + lane; unused slots are KEY_MAX.
+template <int QR>
+struct RegArr {
+  uint64_t v[QR];
+
+  __device__ __forceinline__ void clear() {
+#pragma unroll
+    for (int r = 0; r < QR; ++r) v[r] = KEY_MAX;
+  }
+  // element e (warp-uniform)
+  __device__ __forceinline__ uint64_t get(int e) const {
+    uint64_t x = v[0];
+#pragma unroll
+    for (int r = 1; r < QR; ++r)
+      if ((e >> 5) == r) x = v[r];
+    return __shfl_sync(FULL, x, e & 31);
+  }
+  // remove element 0 (the head), shifting the rest down
+  __device__ __forceinline__ void pop_front(int lane) {
+#pragma unroll
+    for (int r = 0; r < QR; ++r) {
+      uint64_t nxt = (r + 1 < QR) ? __shfl_sync(FULL, v[r + 1 < QR ? r + 1 : r], 0) : KEY_MAX;
+      uint64_t d = __shfl_down_sync(FULL, v[r], 1);
+      v[r] = (lane == 31) ? nxt : d;
+    }
+  }
+  // insert x at its sorted position, capacity L; returns the evicted key
+  // (old element L-1 when the array was full) or KEY_MAX
+  __device__ __forceinline__ uint64_t insert_one(uint64_t x, int L, int lane) {
+    int pos = 0;
+#pragma unroll
+    for (int r = 0; r < QR; ++r) pos += __popc(__ballot_sync(FULL, v[r] < x));
+    const uint64_t evicted = get(L - 1);
+    uint64_t prev[QR];
+#pragma unroll
+    for (int r = 0; r < QR; ++r) {
+      uint64_t up = __shfl_up_sync(FULL, v[r], 1);
+      uint64_t last = (r > 0) ? __shfl_sync(FULL, v[r > 0 ? r - 1 : 0], 31) : KEY_MAX;
+      prev[r] = (lane == 0) ? last : up;
+    }
+#pragma unroll
+    for (int r = 0; r < QR; ++r) {
+      const int e = r * 32 + lane;
+      uint64_t y = (e < pos) ? v[r] : ((e == pos) ? x : prev[r]);
+      v[r] = (e < L) ? y : KEY_MAX;
+    }
+    return (pos < L) ? evicted : KEY_MAX;
+  }
+};
+
+// Bitonic merge of the sorted queue q (QR regs) with 32 keys sorted
+// DESCENDING (one reg): the 32*QR smallest stay in q (ascending) and the rest
+// are returned in `out` (one reg, unordered, KEY_MAX where empty).  Entries of
+// q at positions >= L are also moved out (to out2, one per lane per reg).
+template <int QR>
+__device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int lane, uint64_t& out) {
+  // first half-cleaner of the 64*QR-long bitonic sequence [q asc | MAX.. | s desc]
+  // only touches the last q register (the MAX block pairs with the rest)
+  const uint64_t lo = umin64(q.v[QR - 1], sdesc);
+  out = umax64(q.v[QR - 1], sdesc);
+  q.v[QR - 1] = lo;
+  // the lower half is bitonic: finish the merge (ascending)
+#pragma unroll
+  for (int m = QR / 2; m >= 1; m >>= 1) {
+#pragma unroll
+    for (int r = 0; r < QR; ++r) {
+      if ((r & m) == 0) {
+        uint64_t a = q.v[r], b = q.v[r + m];
+        q.v[r] = umin64(a, b);
+        q.v[r + m] = umax64(a, b);
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 16; j >= 1; j >>= 1) {
+    const bool lower = (lane & j) == 0;
+#pragma unroll
+    for (int r = 0; r < QR; ++r) {
+      uint64_t o = __shfl_xor_sync(FULL, q.v[r], j);
+      q.v[r] = lower ? umin64(q.v[r], o) : umax64(q.v[r], o);
+    }
+  }
+}
+
 // ------------------------------------------------------- bulk distance --
 // §VI: distances of the nc candidates whose ids are in cid[0..nc) (shared).
-// Lane j (< nc) receives candidate j's distance.  NCH = 16 B chunks per lane
-// per row (dpad <= 128 * NCH).
+// Rows are staged R at a time in `stage` by bulk copies; lane j (< nc)
+// receives candidate j's distance.  NCH = 16 B chunks per lane per row.
+template <int NCH>
+struct StageRows {
+  static constexpr int R = (NCH >= 8) ? 4 : (32 / NCH);  // rows per round
+};
+
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
-                                               int lane) {
-  constexpr int R = (NCH >= 8) ? 1 : (8 / NCH);  // rows per batch: 8 LDG.128 in flight
+                                               float* stage, uint64_t* bar, uint32_t& phase,
+                                               int cosine, int lane) {
+  constexpr int R = StageRows<NCH>::R;
   constexpr int LR = Log2<R>::value;
   const int d4 = dpad >> 2;
+  const uint32_t rowbytes = (uint32_t)dpad * 4u;
   float mine = 0.0f;
   for (int b = 0; b < nc; b += R) {
-    float4 x[R][NCH];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      int j = b + r;
-      int id = (j < nc) ? cid[j] : -1;
-      const float4* row = reinterpret_cast<const float4*>(data + (int64_t)(id < 0 ? 0 : id) * dpad);
-#pragma unroll
-      for (int c = 0; c < NCH; ++c) {
-        int idx = c * 32 + lane;
-        if (id >= 0 && idx < d4)
-          x[r][c] = ldg_f4(row + idx);
-        else
-          x[r][c] = make_float4(0.f, 0.f, 0.f, 0.f);
-      }
+    const int rows = min(R, nc - b);
+    // ---- issue: one bulk copy per candidate row, all in flight together
+    fence_proxy_async();
+    if (lane == 0) mbar_arrive_expect_tx(bar, rowbytes * (uint32_t)rows);
+    __syncwarp();
+    if (lane < rows) {
+      const int id = cid[b + lane];
+      bulk_g2s(stage + (size_t)lane * dpad, data + (int64_t)id * dpad, rowbytes, bar);
     }
+    mbar_wait(bar, phase);
+    phase ^= 1u;
+    // ---- compute: lane owns 16 B slices of every staged row
     float part[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       float acc = 0.0f;
+      if (r < rows) {
+        const float4* row = reinterpret_cast<const float4*>(stage + (size_t)r * dpad);
 #pragma unroll
-      for (int c = 0; c < NCH; ++c) {
-        if (METRIC == 0) {
-          float t0 = qv[c].x - x[r][c].x, t1 = qv[c].y - x[r][c].y;
-          float t2 = qv[c].z - x[r][c].z, t3 = qv[c].w - x[r][c].w;
-          acc = fmaf(t0, t0, acc);
-          acc = fmaf(t1, t1, acc);
-          acc = fmaf(t2, t2, acc);
-          acc = fmaf(t3, t3, acc);
-        } else {
-          acc = fmaf(qv[c].x, x[r][c].x, acc);
-          acc = fmaf(qv[c].y, x[r][c].y, acc);
-          acc = fmaf(qv[c].z, x[r][c].z, acc);
-          acc = fmaf(qv[c].w, x[r][c].w, acc);
+        for (int c = 0; c < NCH; ++c) {
+          const int idx = c * 32 + lane;
+          if (idx < d4) {
+            const float4 x = row[idx];
+            if (METRIC == MET_L2) {
+              float t0 = qv[c].x - x.x, t1 = qv[c].y - x.y;
+              float t2 = qv[c].z - x.z, t3 = qv[c].w - x.w;
+              acc = fmaf(t0, t0, acc);
+              acc = fmaf(t1, t1, acc);
+              acc = fmaf(t2, t2, acc);
+              acc = fmaf(t3, t3, acc);
+            } else {
+              acc = fmaf(qv[c].x, x.x, acc);
+              acc = fmaf(qv[c].y, x.y, acc);
+              acc = fmaf(qv[c].z, x.z, acc);
+              acc = fmaf(qv[c].w, x.w, acc);
+            }
+          }
         }
       }
       part[r] = acc;
@@ -279,30 +429,37 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     float tot = transpose_reduce<R>(part, lane);
     float got = __shfl_sync(FULL, tot, ((lane - b) & (R - 1)) << (5 - LR));
     if (lane >= b && lane < b + R) mine = got;
+    __syncwarp();
   }
-  if (METRIC == 1) mine = -mine;        // inner product: -<q,x>
-  if (METRIC == 2) mine = 1.0f - mine;  // cosine on unit rows: 1 - cos
+  if (METRIC == MET_DOT) mine = cosine ? 1.0f - mine : -mine;  // 1 - cos / -<q,x>
   return mine;
 }
 
 // ---------------------------------------------------------- the kernel --
-template <int NCH, int METRIC, bool BLOOM>
+// QR > 0: q / topk in registers (queue_len <= 32*QR); QR == 0: shared memory.
+template <int NCH, int METRIC, bool BLOOM, int QR>
 __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
-  extern __shared__ __align__(16) unsigned char smem[];
+  extern __shared__ __align__(128) unsigned char smem[];
+  constexpr int R = StageRows<NCH>::R;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
-  uint64_t* qa = reinterpret_cast<uint64_t*>(base);  // q, current buffer
-  uint64_t* qb = qa + L;                              // q, next buffer
-  uint64_t* tk = qb + L;                              // topk, sorted ascending
-  uint64_t* stage = tk + L;                           // 32 sorted new keys
-  int* cid = reinterpret_cast<int*>(stage + 32);      // 32 candidate ids
-  int* table = cid + 32;                              // visited
+  float* stage = reinterpret_cast<float*>(base);                       // R rows
+  uint64_t* bar = reinterpret_cast<uint64_t*>(base + (size_t)R * a.dpad * 4);
+  int* cid = reinterpret_cast<int*>(bar + 2);                           // 32 ids
+  uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
+  uint64_t* qa = keys32 + 32;                                           // QR == 0 only
+  uint64_t* qb = qa + (QR == 0 ? L : 0);
+  uint64_t* tk = qb + (QR == 0 ? L : 0);
+  int* table = reinterpret_cast<int*>(tk + (QR == 0 ? L : 0));
   const int tslots = BLOOM ? ((1 << a.table_log2) >> 5) : (1 << a.table_log2);
   HashSet hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};
   const unsigned lt = lanemask_lt();
+  if (lane == 0) mbar_init(bar);
+  __syncwarp();
+  uint32_t phase = 0;
 
   while (true) {
     int qi = 0;
@@ -325,7 +482,7 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       qv[c] = make_float4(v0, v1, v2, v3);
     }
     bad = __any_sync(FULL, bad);
-    if (METRIC == 2) {
+    if (METRIC == MET_DOT && a.cosine) {
       float s = 0.f;
 #pragma unroll
       for (int c = 0; c < NCH; ++c)
@@ -360,19 +517,29 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
     for (int i = lane; i < tslots; i += 32) table[i] = BLOOM ? 0 : EMPTY;
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, lane);
-    int used = 0;
+    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, bar, phase,
+                                                a.cosine, lane);
+    const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     if (lane == 0) {
-      qa[0] = make_key(de, a.entry);
       if (BLOOM)
         bs.insert(a.entry);
       else
         hs.insert(a.entry);
     }
-    used = 1;
+    int used = 1;
+    RegArr<QR == 0 ? 1 : QR> q, tk_r;
+    q.clear();
+    tk_r.clear();
+    if (QR > 0) {
+      if (lane == 0) q.v[0] = ke;
+    } else if (lane == 0) {
+      qa[0] = ke;
+    }
     int qsize = 1, tsize = 0;
     int n_dist = 1, n_exp = 0, iters = 0;
     bool capped = false;
+    // adjacency row of the next head, prefetched (lane j holds slot j)
+    int adjv = (lane < a.degree) ? __ldg(a.adj + (int64_t)a.entry * a.degree + lane) : -1;
     __syncwarp();
 
     while (qsize > 0) {
@@ -382,60 +549,84 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       }
       ++iters;
       // ---- a3: pop / terminate / topk update (Alg. 1 lines 3-8)
-      const uint64_t now = qa[0];
-      const bool full = (tsize == L);
-      if (full && tk[L - 1] < now) break;
-      const uint64_t evicted = full ? tk[L - 1] : KEY_MAX;
-      int pos = 0;
-      for (int b0 = 0; b0 < tsize; b0 += 32) {
-        int i = b0 + lane;
-        pos += __popc(__ballot_sync(FULL, i < tsize && tk[i] < now));
+      uint64_t now, tmax;
+      if (QR > 0) {
+        now = __shfl_sync(FULL, q.v[0], 0);
+        tmax = tk_r.get(L - 1);  // KEY_MAX unless topk is full
+      } else {
+        now = qa[0];
+        tmax = (tsize == L) ? tk[L - 1] : KEY_MAX;
       }
-      const int newsize = full ? L : tsize + 1;
-      for (int b0 = ((newsize - 1) >> 5) << 5; b0 >= ((pos >> 5) << 5); b0 -= 32) {
-        int i = b0 + lane;
-        uint64_t val = 0;
-        bool w = false;
-        if (i > pos && i < newsize) {
-          val = tk[i - 1];
-          w = true;
-        } else if (i == pos) {
-          val = now;
-          w = true;
+      if (tmax < now) break;  // topk full and its max beats now (lines 4-5)
+      uint64_t evicted = KEY_MAX;
+      if (QR > 0) {
+        evicted = tk_r.insert_one(now, L, lane);
+        q.pop_front(lane);
+      } else {
+        evicted = (tsize == L) ? tk[L - 1] : KEY_MAX;
+        int pos = 0;
+        for (int b0 = 0; b0 < tsize; b0 += 32) {
+          int i = b0 + lane;
+          pos += __popc(__ballot_sync(FULL, i < tsize && tk[i] < now));
         }
-        __syncwarp();
-        if (w) tk[i] = val;
+        const int newsize = min(tsize + 1, L);
+        for (int b0 = ((newsize - 1) >> 5) << 5; b0 >= ((pos >> 5) << 5); b0 -= 32) {
+          int i = b0 + lane;
+          uint64_t val = 0;
+          bool w = false;
+          if (i > pos && i < newsize) {
+            val = tk[i - 1];
+            w = true;
+          } else if (i == pos) {
+            val = now;
+            w = true;
+          }
+          __syncwarp();
+          if (w) tk[i] = val;
+        }
       }
-      tsize = newsize;
-      if (!BLOOM && full && lane == 0) hs.erase(key_id(evicted));  // §IV-E
+      tsize = min(tsize + 1, L);
+      if (!BLOOM && evicted != KEY_MAX && lane == 0) hs.erase(key_id(evicted));  // §IV-E
       __syncwarp();
-      const uint64_t* A = qa + 1;  // q after the pop
-      const int na = qsize - 1;
+      const int na = qsize - 1;  // q after the pop
+      const uint64_t* A = qa + 1;
 
       // ---- a4: candidate locating (§V)
-      const int nowid = key_id(now);
-      int v = (lane < a.degree) ? __ldg(a.adj + (int64_t)nowid * a.degree + lane) : -1;
-      unsigned grp = __match_any_sync(FULL, v);
-      bool keep = (v >= 0) && ((grp & lt) == 0);
+      int v = adjv;
+      bool keep = v >= 0;
+      if (a.dedup) {
+        unsigned grp = __match_any_sync(FULL, v);
+        keep = keep && ((grp & lt) == 0);
+      }
       if (keep) keep = BLOOM ? !bs.contains(v) : !hs.contains(v);
-      unsigned km = __ballot_sync(FULL, keep);
+      const unsigned km = __ballot_sync(FULL, keep);
       const int nc = __popc(km);
       if (keep) cid[__popc(km & lt)] = v;
       __syncwarp();
 
       // ---- a5: bulk distance computation (§VI)
-      float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, lane);
+      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, bar,
+                                                    phase, a.cosine, lane);
       n_dist += nc;
       n_exp += 1;
 
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cid[lane] : -1;
       uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
-      const uint64_t thr = (tsize == L) ? tk[L - 1] : KEY_MAX;
+      const uint64_t thr = (tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
       const bool sel = (lane < nc) && key < thr;  // selected insertion
-      const unsigned sm = __ballot_sync(FULL, sel);
-      const int ns = __popc(sm);
+      const int ns = __popc(__ballot_sync(FULL, sel));
       if (!sel) key = KEY_MAX;
+      // prefetch the adjacency row of the next head = min(q head, best new key)
+      {
+        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na > 0 ? A[0] : KEY_MAX);
+        uint64_t nxt = umin64(qhead, warp_min_key(key));
+        if (nxt != KEY_MAX && lane < a.degree)
+          adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
+        else
+          adjv = -1;
+      }
+      // visited insert of the selected candidates
       if (BLOOM) {
         if (sel) bs.insert(myid);
       } else {
@@ -443,59 +634,93 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
           // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
           for (int i = lane; i < tslots; i += 32) table[i] = EMPTY;
           __syncwarp();
-          for (int i = lane; i < na; i += 32) hs.insert(key_id(A[i]));
-          for (int i = lane; i < tsize; i += 32) hs.insert(key_id(tk[i]));
+          if (QR > 0) {
+#pragma unroll
+            for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+              if (q.v[r] != KEY_MAX) hs.insert(key_id(q.v[r]));
+              if (tk_r.v[r] != KEY_MAX) hs.insert(key_id(tk_r.v[r]));
+            }
+          } else {
+            for (int i = lane; i < na; i += 32) hs.insert(key_id(A[i]));
+            for (int i = lane; i < tsize; i += 32) hs.insert(key_id(tk[i]));
+          }
           used = na + tsize;
           __syncwarp();
         }
-        bool took = sel ? hs.insert(myid) : false;
+        const bool took = sel ? hs.insert(myid) : false;
         used += __popc(__ballot_sync(FULL, took));
       }
-      key = bitonic_sort32(key, lane);
-      stage[lane] = key;
       __syncwarp();
-      // merge q (A, na) with the selected keys (stage, ns) into qb, keep L
-      for (int i = lane; i < na; i += 32) {
-        uint64_t x = A[i];
-        int p = i + count_below(stage, ns, x);
-        if (p < L)
-          qb[p] = x;
-        else if (!BLOOM)
-          hs.erase(key_id(x));
-      }
-      if (lane < ns) {
-        int p = lane + count_below(A, na, key);
-        if (p < L)
-          qb[p] = key;
-        else if (!BLOOM)
-          hs.erase(key_id(key));
+      if (QR > 0) {
+        // merge the selected keys into q; evict beyond L (§IV-C) and delete (§IV-E)
+        const uint64_t sdesc = bitonic_sort32<true>(key, lane);
+        uint64_t out;
+        merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
+#pragma unroll
+        for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+          if (r * 32 + lane >= L) {
+            if (!BLOOM && q.v[r] != KEY_MAX) hs.erase(key_id(q.v[r]));
+            q.v[r] = KEY_MAX;
+          }
+        }
+        if (!BLOOM && out != KEY_MAX) hs.erase(key_id(out));
+      } else {
+        key = bitonic_sort32<false>(key, lane);
+        keys32[lane] = key;
+        __syncwarp();
+        for (int i = lane; i < na; i += 32) {
+          uint64_t x = A[i];
+          int p = i + count_below(keys32, ns, x);
+          if (p < L)
+            qb[p] = x;
+          else if (!BLOOM)
+            hs.erase(key_id(x));
+        }
+        if (lane < ns) {
+          int p = lane + count_below(A, na, key);
+          if (p < L)
+            qb[p] = key;
+          else if (!BLOOM)
+            hs.erase(key_id(key));
+        }
+        uint64_t* t = qa;
+        qa = qb;
+        qb = t;
       }
       qsize = min(na + ns, L);
-      uint64_t* t = qa;
-      qa = qb;
-      qb = t;
       __syncwarp();
     }
 
     // ---- a7: output the first K of topk (Alg. 1 line 17)
-    for (int i = lane; i < a.K; i += 32) {
-      if (i < tsize) {
-        uint64_t k = tk[i];
-        ids_o[i] = key_id(k) + a.id_offset;
-        dists_o[i] = ord2f((uint32_t)(k >> 32));
-      } else {
-        ids_o[i] = -1;
-        dists_o[i] = __int_as_float(0x7f800000);
+    if (QR > 0) {
+#pragma unroll
+      for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+        const int i = r * 32 + lane;
+        if (i < a.K) {
+          uint64_t k = tk_r.v[r];
+          ids_o[i] = (k != KEY_MAX) ? key_id(k) + a.id_offset : -1;
+          dists_o[i] = (k != KEY_MAX) ? ord2f((uint32_t)(k >> 32)) : __int_as_float(0x7f800000);
+        }
       }
+    } else {
+      for (int i = lane; i < a.K; i += 32) {
+        if (i < tsize) {
+          uint64_t k = tk[i];
+          ids_o[i] = key_id(k) + a.id_offset;
+          dists_o[i] = ord2f((uint32_t)(k >> 32));
+        } else {
+          ids_o[i] = -1;
+          dists_o[i] = __int_as_float(0x7f800000);
+        }
+      }
+      qa = keys32 + 32;
+      qb = qa + L;
     }
     if (a.counters_out && lane == 0) {
       a.counters_out[2 * (int64_t)qi] = n_dist;
       a.counters_out[2 * (int64_t)qi + 1] = n_exp;
     }
     if (capped && lane == 0) atomicOr(a.status, STATUS_ITER_CAP);
-    // restore buffer roles so the next query starts from the block's layout
-    qa = reinterpret_cast<uint64_t*>(base);
-    qb = qa + L;
     __syncwarp();
   }
 }

@@ -25,6 +25,7 @@ struct song_index {
   int32_t* d_adj = nullptr;
   unsigned* d_ticket = nullptr;
   int* d_status = nullptr;
+  int dedup = 1;                       // some adjacency row repeats an id
   cudaStream_t stream = nullptr;       // owned; used by song_search
   cudaStream_t last_stream = nullptr;  // stream of the last search
   // scratch for the host-buffer entry point
@@ -77,6 +78,22 @@ __global__ void validate_kernel(const float* __restrict__ v, int64_t nv,
     local += (a < -1 || a >= n);
   }
   if (local) atomicAdd(bad, local);
+}
+
+// Does any adjacency row list an id twice?  (If not, the search kernel skips
+// the in-row de-duplication of reading A7.)
+__global__ void dup_check_kernel(const int32_t* __restrict__ adj, int64_t n, int degree,
+                                 int* any_dup) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n;
+       r += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    int v = lane < degree ? adj[r * degree + lane] : -1;
+    unsigned lt;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+    unsigned grp = __match_any_sync(0xffffffffu, v);
+    bool dup = v >= 0 && (grp & lt) != 0;
+    if (__any_sync(0xffffffffu, dup) && lane == 0) atomicOr(any_dup, 1);
+  }
 }
 
 // Cosine: rows are L2-normalised once at index creation so the search
@@ -138,13 +155,15 @@ int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* a
   return SONG_OK;
 }
 
-// per-warp shared memory of the search kernel
+// per-warp shared memory of the search kernel (DESIGN.md §4)
 struct Shape {
   int table_log2;
   int warp_bytes;
+  int qr;  // register queue width (L <= 32*qr), 0 = shared-memory queues
+  int nch;
 };
 
-Shape search_shape(int L, bool bloom, int bloom_log2_bits) {
+Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   Shape s;
   int tbytes;
   if (bloom) {
@@ -156,15 +175,19 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits) {
     s.table_log2 = next_pow2_log2(2ll * (2 * L + 32));
     tbytes = (1 << s.table_log2) * 4;
   }
-  s.warp_bytes = 3 * L * 8 + 32 * 8 + 32 * 4 + tbytes;
-  s.warp_bytes = (s.warp_bytes + 15) & ~15;
+  s.nch = (dpad + 127) / 128;
+  s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
+  const int rows = s.nch >= 8 ? 4 : 32 / s.nch;  // StageRows<NCH>::R
+  s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
+  s.warp_bytes = rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 : 0) + tbytes;
+  s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;
 }
 
-template <int NCH, int METRIC, bool BLOOM>
+template <int NCH, int METRIC, bool BLOOM, int QR>
 int launch_t(const song::SearchArgs& a, int warps, int blocks_per_sm, int num_sms,
              cudaStream_t st) {
-  auto kern = song::song_search_kernel<NCH, METRIC, BLOOM>;
+  auto kern = song::song_search_kernel<NCH, METRIC, BLOOM, QR>;
   const size_t smem = (size_t)a.warp_smem_bytes * warps;
   CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int fit = 0;
@@ -179,17 +202,24 @@ int launch_t(const song::SearchArgs& a, int warps, int blocks_per_sm, int num_sm
   return SONG_OK;
 }
 
+template <int NCH, int METRIC, bool BLOOM>
+int launch_q(const song::SearchArgs& a, int qr, int warps, int bps, int sms, cudaStream_t st) {
+  switch (qr) {
+    case 1: return launch_t<NCH, METRIC, BLOOM, 1>(a, warps, bps, sms, st);
+    case 2: return launch_t<NCH, METRIC, BLOOM, 2>(a, warps, bps, sms, st);
+    case 4: return launch_t<NCH, METRIC, BLOOM, 4>(a, warps, bps, sms, st);
+    default: return launch_t<NCH, METRIC, BLOOM, 0>(a, warps, bps, sms, st);
+  }
+}
+
 template <int NCH>
-int launch_m(const song::SearchArgs& a, int metric, bool bloom, int warps, int bps, int sms,
-             cudaStream_t st) {
+int launch_m(const song::SearchArgs& a, int metric, bool bloom, int qr, int warps, int bps,
+             int sms, cudaStream_t st) {
   if (metric == SONG_L2)
-    return bloom ? launch_t<NCH, 0, true>(a, warps, bps, sms, st)
-                 : launch_t<NCH, 0, false>(a, warps, bps, sms, st);
-  if (metric == SONG_IP)
-    return bloom ? launch_t<NCH, 1, true>(a, warps, bps, sms, st)
-                 : launch_t<NCH, 1, false>(a, warps, bps, sms, st);
-  return bloom ? launch_t<NCH, 2, true>(a, warps, bps, sms, st)
-               : launch_t<NCH, 2, false>(a, warps, bps, sms, st);
+    return bloom ? launch_q<NCH, song::MET_L2, true>(a, qr, warps, bps, sms, st)
+                 : launch_q<NCH, song::MET_L2, false>(a, qr, warps, bps, sms, st);
+  return bloom ? launch_q<NCH, song::MET_DOT, true>(a, qr, warps, bps, sms, st)
+               : launch_q<NCH, song::MET_DOT, false>(a, qr, warps, bps, sms, st);
 }
 
 int check_params(const song_index* ix, const song_search_params* p) {
@@ -227,8 +257,10 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.degree = ix->degree;
   a.K = p->K;
   a.L = p->queue_len;
+  a.cosine = ix->metric == SONG_COSINE;
+  a.dedup = ix->dedup;
   const bool bloom = p->visited == SONG_VISITED_BLOOM;
-  Shape sh = search_shape(p->queue_len, bloom, p->bloom_log2_bits);
+  Shape sh = search_shape(p->queue_len, bloom, p->bloom_log2_bits, ix->dpad);
   a.table_log2 = sh.table_log2;
   a.warp_smem_bytes = sh.warp_bytes;
   a.entry = p->entry;
@@ -240,14 +272,30 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
     return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
                 p->queue_len, sh.warp_bytes);
   ix->last_stream = st;
-  const int nch = (ix->dpad + 127) / 128;
-  if (nch <= 1) return launch_m<1>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
-  if (nch <= 2) return launch_m<2>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
-  if (nch <= 4) return launch_m<4>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
-  return launch_m<8>(a, ix->metric, bloom, warps, p->blocks_per_sm, ix->num_sms, st);
+  const int m = ix->metric, qr = sh.qr, bps = p->blocks_per_sm, sms = ix->num_sms;
+  switch (sh.nch) {
+    case 1: return launch_m<1>(a, m, bloom, qr, warps, bps, sms, st);
+    case 2: return launch_m<2>(a, m, bloom, qr, warps, bps, sms, st);
+    case 4: return launch_m<4>(a, m, bloom, qr, warps, bps, sms, st);
+    default: return launch_m<8>(a, m, bloom, qr, warps, bps, sms, st);
+  }
 }
 
 int finish_create(song_index* ix, cudaStream_t st) {
+  {
+    int* d_dup = nullptr;
+    CUDA_TRY(cudaMalloc(&d_dup, sizeof(int)));
+    CUDA_TRY(cudaMemsetAsync(d_dup, 0, sizeof(int), st));
+    int blocks = (int)std::min<int64_t>((ix->n + 7) / 8, 65535);
+    dup_check_kernel<<<blocks, 256, 0, st>>>(ix->d_adj, ix->n, ix->degree, d_dup);
+    int dup = 1;
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&dup, d_dup, sizeof(int), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFree(d_dup);
+    if (e != cudaSuccess) return fail(SONG_ECUDA, "dup check: %s", cudaGetErrorString(e));
+    ix->dedup = dup;
+  }
   if (ix->metric == SONG_COSINE) {
     int blocks = (int)std::min<int64_t>((ix->n + 7) / 8, 65535);
     normalize_rows_kernel<<<blocks, 256, 0, st>>>(ix->d_data, ix->n, ix->dpad);
