@@ -11,4 +11,4 @@ timeout 600 ncu --nvtx --nvtx-include "song_timed/" --metrics gpu__time_duration
 timeout 900 ncu --nvtx --nvtx-include "song_timed/" --set full --clock-control none --import-source on \
   -k regex:song_search -c 1 -o gpurun_out/${TAG}_full \
   python bench.py $ARGS --cache /tmp/song_w.pt --profile --steps 1 --warmup 1 > gpurun_out/${TAG}_full.log 2>&1
-tail -3 gpurun_out/${TAG}_*.log
+for f in gpurun_out/${TAG}_*.log; do tail -n 3 $f; done

@@ -139,15 +139,19 @@ __device__ __forceinline__ void fence_proxy_async() {
 }
 
 // ---------------------------------------------------------------- visited --
-// Open-addressing hash in shared memory, linear probing; every lane
-// runs its own probe sequence so up to 32 operations proceed in parallel.
+// Open-addressing hash in shared memory, linear probing.  Every lane
+// runs its own probe sequence, so up to 32 operations proceed in parallel;
+// all loops are warp-collective (trip count decided by __any_sync) so the
+// warp stays converged for the shuffles that follow.
+#ifdef SONG_OLD_HASH
 struct HashSet {
   int* slot;
   int log2;
   __device__ __forceinline__ unsigned home(int v) const {
     return ((uint32_t)v * 0x9E3779B1u) >> (32 - log2);
   }
-  __device__ __forceinline__ bool contains(int v) const {
+  __device__ __forceinline__ bool contains(int v, bool act) const {
+    if (!act) return false;
     unsigned mask = (1u << log2) - 1, h = home(v);
     while (true) {
       int s = slot[h];
@@ -156,32 +160,99 @@ struct HashSet {
       h = (h + 1) & mask;
     }
   }
-  // returns true when an EMPTY slot was consumed
-  __device__ __forceinline__ bool insert(int v) {
+  __device__ __forceinline__ bool insert(int v, bool act) {
+    bool r = false;
+    if (act) {
     unsigned mask = (1u << log2) - 1, h = home(v);
     while (true) {
       int s = slot[h];
       if (s == EMPTY || s == TOMB) {
         int old = atomicCAS(&slot[h], s, v);
-        if (old == s) return s == EMPTY;
-        continue;  // lost the race for this slot: re-read it
+        if (old == s) { r = (s == EMPTY); break; }
+        continue;
       }
       h = (h + 1) & mask;
     }
+    }
+    __syncwarp();
+    return r;
   }
-  __device__ __forceinline__ void erase(int v) {
+  __device__ __forceinline__ void erase(int v, bool act) {
+    if (act) {
     unsigned mask = (1u << log2) - 1, h = home(v);
     while (true) {
       int s = slot[h];
-      if (s == v) {
-        slot[h] = TOMB;
-        return;
-      }
-      if (s == EMPTY) return;
+      if (s == v) { slot[h] = TOMB; break; }
+      if (s == EMPTY) break;
       h = (h + 1) & mask;
+    }
+    }
+    __syncwarp();
+  }
+};
+#else
+struct HashSet {
+  int* slot;
+  int log2;
+  __device__ __forceinline__ unsigned home(int v) const {
+    return ((uint32_t)v * 0x9E3779B1u) >> (32 - log2);
+  }
+  // membership of v for lanes with act; result false elsewhere
+  __device__ __forceinline__ bool contains(int v, bool act) const {
+    const unsigned mask = (1u << log2) - 1;
+    unsigned h = home(v);
+    bool found = false;
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const int s = slot[h];
+        found = (s == v);
+        act = !found && s != EMPTY;
+        h = (h + 1) & mask;
+      }
+    }
+    return found;
+  }
+  // insert v (not present) for lanes with act; true when an EMPTY slot was used
+  __device__ __forceinline__ bool insert(int v, bool act) {
+    const unsigned mask = (1u << log2) - 1;
+    unsigned h = home(v);
+    bool took_empty = false;
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const int s = slot[h];
+        if (s == EMPTY || s == TOMB) {
+          const int old = atomicCAS(&slot[h], s, v);
+          if (old == s) {
+            act = false;
+            took_empty = (s == EMPTY);
+          }  // else: lost the race for this slot, re-read it
+        } else {
+          h = (h + 1) & mask;
+        }
+      }
+    }
+    return took_empty;
+  }
+  // delete v (present) for lanes with act (§IV-E): the slot becomes a tombstone
+  __device__ __forceinline__ void erase(int v, bool act) {
+    const unsigned mask = (1u << log2) - 1;
+    unsigned h = home(v);
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const int s = slot[h];
+        if (s == v) {
+          slot[h] = TOMB;
+          act = false;
+        } else if (s == EMPTY) {
+          act = false;
+        } else {
+          h = (h + 1) & mask;
+        }
+      }
     }
   }
 };
+#endif
 
 // Bloom filter with the k = 7 double-hashing spec of reading A8:
 // bit_i = (h1 + i*h2) mod m, h1 = fmix32(id), h2 = fmix32(id ^ 0x5bd1e995) | 1.
@@ -197,24 +268,28 @@ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
 struct BloomSet {
   uint32_t* word;
   int log2;  // m = 2^log2 bits
-  __device__ __forceinline__ bool contains(int v) const {
-    uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
-    uint32_t mask = (1u << log2) - 1;
+  __device__ __forceinline__ bool contains(int v, bool act) const {
+    const uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
+    const uint32_t mask = (1u << log2) - 1;
+    bool all = true;
 #pragma unroll
     for (int i = 0; i < 7; ++i) {
-      uint32_t b = (h1 + (uint32_t)i * h2) & mask;
-      if (!((word[b >> 5] >> (b & 31)) & 1u)) return false;
+      const uint32_t b = (h1 + (uint32_t)i * h2) & mask;
+      all = all && (act ? ((word[b >> 5] >> (b & 31)) & 1u) : 0u);
     }
-    return true;
+    return act && all;
   }
-  __device__ __forceinline__ void insert(int v) {
-    uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
-    uint32_t mask = (1u << log2) - 1;
+  __device__ __forceinline__ void insert(int v, bool act) {
+    const uint32_t h1 = fmix32((uint32_t)v), h2 = fmix32((uint32_t)v ^ 0x5bd1e995u) | 1u;
+    const uint32_t mask = (1u << log2) - 1;
+    if (act) {
 #pragma unroll
-    for (int i = 0; i < 7; ++i) {
-      uint32_t b = (h1 + (uint32_t)i * h2) & mask;
-      atomicOr(&word[b >> 5], 1u << (b & 31));
+      for (int i = 0; i < 7; ++i) {
+        const uint32_t b = (h1 + (uint32_t)i * h2) & mask;
+        atomicOr(&word[b >> 5], 1u << (b & 31));
+      }
     }
+    __syncwarp();
   }
 };
 
@@ -235,14 +310,12 @@ __device__ __forceinline__ uint64_t bitonic_sort32(uint64_t key, int lane) {
 }
 
 // number of elements of sorted a[0..n) strictly below x
+// (branch-free: the trip count depends only on the warp-uniform n)
 __device__ __forceinline__ int count_below(const uint64_t* a, int n, uint64_t x) {
-  int lo = 0, hi = n;
-  while (lo < hi) {
-    int mid = (lo + hi) >> 1;
-    if (a[mid] < x)
-      lo = mid + 1;
-    else
-      hi = mid;
+  int lo = 0;
+  for (int step = 1 << (31 - __clz(n | 1)); step > 0; step >>= 1) {
+    const int j = lo + step - 1;
+    lo = (j < n && a[j] < x) ? lo + step : lo;
   }
   return lo;
 }
@@ -367,69 +440,133 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
 
 // ------------------------------------------------------- bulk distance --
 // §VI: distances of the nc candidates whose ids are in cid[0..nc) (shared).
-// Rows are staged R at a time in `stage` by bulk copies; lane j (< nc)
-// receives candidate j's distance.  NCH = 16 B chunks per lane per row.
+// Rows are staged R at a time in `stage` by cp.async (LDGSTS, 16 B per lane
+// per row, L1-bypassing): every row of the round is in flight at once with no
+// register cost, then each lane reads back only its own 16 B slices (no
+// cross-lane hazard) and a transposed butterfly reduces the R partial sums.
+// Lane j (< nc) receives candidate j's distance.  NCH = 16 B chunks per lane.
 template <int NCH>
 struct StageRows {
   static constexpr int R = (NCH >= 8) ? 4 : (32 / NCH);  // rows per round
 };
 
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src)
+               : "memory");
+}
+
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.wait_all;" ::: "memory");
+}
+
+// packed fp32x2 arithmetic (sm_100: FADD2 / FFMA2)
+__device__ __forceinline__ uint64_t f2pack(float lo, float hi) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+
+__device__ __forceinline__ float f2sum(uint64_t v) {
+  float lo, hi;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+  return lo + hi;
+}
+
+template <int METRIC>
+__device__ __forceinline__ uint64_t acc4(uint64_t acc, uint64_t q01, uint64_t q23, float4 x) {
+#ifdef SONG_SCALAR_FMA
+  float a0, a1, q0, q1, q2, q3;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a0), "=f"(a1) : "l"(acc));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(q0), "=f"(q1) : "l"(q01));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(q2), "=f"(q3) : "l"(q23));
+  if (METRIC == MET_L2) {
+    float t0 = q0 - x.x, t1 = q1 - x.y, t2 = q2 - x.z, t3 = q3 - x.w;
+    a0 = fmaf(t0, t0, a0); a1 = fmaf(t1, t1, a1); a0 = fmaf(t2, t2, a0); a1 = fmaf(t3, t3, a1);
+  } else {
+    a0 = fmaf(q0, x.x, a0); a1 = fmaf(q1, x.y, a1); a0 = fmaf(q2, x.z, a0); a1 = fmaf(q3, x.w, a1);
+  }
+  return f2pack(a0, a1);
+#endif
+  const uint64_t x01 = f2pack(x.x, x.y), x23 = f2pack(x.z, x.w);
+  if (METRIC == MET_L2) {
+    uint64_t d01, d23;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d01) : "l"(q01), "l"(x01));
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d23) : "l"(q23), "l"(x23));
+    asm("fma.rn.f32x2 %0, %1, %1, %0;" : "+l"(acc) : "l"(d01));
+    asm("fma.rn.f32x2 %0, %1, %1, %0;" : "+l"(acc) : "l"(d23));
+  } else {
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(q01), "l"(x01));
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(q23), "l"(x23));
+  }
+  return acc;
+}
+
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
-                                               float* stage, uint64_t* bar, uint32_t& phase,
-                                               int cosine, int lane) {
+                                               float* stage, int cosine, int lane) {
   constexpr int R = StageRows<NCH>::R;
   constexpr int LR = Log2<R>::value;
+  constexpr int G = R < 8 ? R : 8;  // rows per uniform compute group
   const int d4 = dpad >> 2;
-  const uint32_t rowbytes = (uint32_t)dpad * 4u;
   float mine = 0.0f;
+  uint64_t q01[NCH], q23[NCH];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    q01[c] = f2pack(qv[c].x, qv[c].y);
+    q23[c] = f2pack(qv[c].z, qv[c].w);
+  }
   for (int b = 0; b < nc; b += R) {
     const int rows = min(R, nc - b);
-    // ---- issue: one bulk copy per candidate row, all in flight together
-    fence_proxy_async();
-    if (lane == 0) mbar_arrive_expect_tx(bar, rowbytes * (uint32_t)rows);
-    __syncwarp();
-    if (lane < rows) {
-      const int id = cid[b + lane];
-      bulk_g2s(stage + (size_t)lane * dpad, data + (int64_t)id * dpad, rowbytes, bar);
-    }
-    mbar_wait(bar, phase);
-    phase ^= 1u;
-    // ---- compute: lane owns 16 B slices of every staged row
-    float part[R];
+    // ---- issue: every row of the round in flight at once
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      float acc = 0.0f;
       if (r < rows) {
-        const float4* row = reinterpret_cast<const float4*>(stage + (size_t)r * dpad);
+        const float4* src = reinterpret_cast<const float4*>(data + (int64_t)cid[b + r] * dpad);
+        float4* dst = reinterpret_cast<float4*>(stage + (size_t)r * dpad);
 #pragma unroll
         for (int c = 0; c < NCH; ++c) {
           const int idx = c * 32 + lane;
-          if (idx < d4) {
-            const float4 x = row[idx];
-            if (METRIC == MET_L2) {
-              float t0 = qv[c].x - x.x, t1 = qv[c].y - x.y;
-              float t2 = qv[c].z - x.z, t3 = qv[c].w - x.w;
-              acc = fmaf(t0, t0, acc);
-              acc = fmaf(t1, t1, acc);
-              acc = fmaf(t2, t2, acc);
-              acc = fmaf(t3, t3, acc);
-            } else {
-              acc = fmaf(qv[c].x, x.x, acc);
-              acc = fmaf(qv[c].y, x.y, acc);
-              acc = fmaf(qv[c].z, x.z, acc);
-              acc = fmaf(qv[c].w, x.w, acc);
-            }
-          }
+          if (idx < d4) cp_async16(dst + idx, src + idx);
         }
       }
-      part[r] = acc;
     }
+    cp_async_wait_all();
+    // ---- compute: lane owns its 16 B slices of every staged row
+    float part[R];
+#pragma unroll
+    for (int g = 0; g < R; g += G) {
+      if (g < rows) {
+#pragma unroll
+        for (int r = g; r < g + G; ++r) {
+          const float4* row = reinterpret_cast<const float4*>(stage + (size_t)r * dpad);
+          uint64_t acc = 0;
+#pragma unroll
+          for (int c = 0; c < NCH; ++c) {
+            const int idx = c * 32 + lane;
+            if (idx < d4) acc = acc4<METRIC>(acc, q01[c], q23[c], row[idx]);
+          }
+          part[r] = f2sum(acc);
+        }
+      } else {
+#pragma unroll
+        for (int r = g; r < g + G; ++r) part[r] = 0.0f;
+      }
+    }
+#ifdef SONG_DEBUG
+    if (lane < 2) {
+      for (int r = 0; r < rows; ++r) {
+        const float4 x = reinterpret_cast<const float4*>(stage + (size_t)r * dpad)[lane];
+        printf("bd lane %d row %d id %d x %f %f %f %f q %f part %f\n", lane, r, cid[b + r], x.x, x.y, x.z, x.w, qv[0].x, part[r]);
+      }
+    }
+#endif
     float tot = transpose_reduce<R>(part, lane);
+#ifdef SONG_DEBUG
+    if (lane < 4) printf("bd lane %d tot %f\n", lane, tot);
+#endif
     float got = __shfl_sync(FULL, tot, ((lane - b) & (R - 1)) << (5 - LR));
     if (lane >= b && lane < b + R) mine = got;
-    __syncwarp();
   }
   if (METRIC == MET_DOT) mine = cosine ? 1.0f - mine : -mine;  // 1 - cos / -<q,x>
   return mine;
@@ -446,8 +583,7 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
   float* stage = reinterpret_cast<float*>(base);                       // R rows
-  uint64_t* bar = reinterpret_cast<uint64_t*>(base + (size_t)R * a.dpad * 4);
-  int* cid = reinterpret_cast<int*>(bar + 2);                           // 32 ids
+  int* cid = reinterpret_cast<int*>(base + (size_t)R * a.dpad * 4 + 16);  // 32 ids
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
   uint64_t* qa = keys32 + 32;                                           // QR == 0 only
   uint64_t* qb = qa + (QR == 0 ? L : 0);
@@ -457,9 +593,6 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
   HashSet hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};
   const unsigned lt = lanemask_lt();
-  if (lane == 0) mbar_init(bar);
-  __syncwarp();
-  uint32_t phase = 0;
 
   while (true) {
     int qi = 0;
@@ -517,15 +650,12 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
     for (int i = lane; i < tslots; i += 32) table[i] = BLOOM ? 0 : EMPTY;
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, bar, phase,
-                                                a.cosine, lane);
+    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, a.cosine, lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
-    if (lane == 0) {
-      if (BLOOM)
-        bs.insert(a.entry);
-      else
-        hs.insert(a.entry);
-    }
+    if (BLOOM)
+      bs.insert(a.entry, lane == 0);
+    else
+      hs.insert(a.entry, lane == 0);
     int used = 1;
     RegArr<QR == 0 ? 1 : QR> q, tk_r;
     q.clear();
@@ -586,7 +716,7 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
         }
       }
       tsize = min(tsize + 1, L);
-      if (!BLOOM && evicted != KEY_MAX && lane == 0) hs.erase(key_id(evicted));  // §IV-E
+      if (!BLOOM) hs.erase(key_id(evicted), evicted != KEY_MAX && lane == 0);  // §IV-E
       __syncwarp();
       const int na = qsize - 1;  // q after the pop
       const uint64_t* A = qa + 1;
@@ -598,15 +728,17 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
         unsigned grp = __match_any_sync(FULL, v);
         keep = keep && ((grp & lt) == 0);
       }
-      if (keep) keep = BLOOM ? !bs.contains(v) : !hs.contains(v);
+      // (called by every lane: the probe loops are warp-collective)
+      const bool seen = BLOOM ? bs.contains(v, keep) : hs.contains(v, keep);
+      keep = keep && !seen;
       const unsigned km = __ballot_sync(FULL, keep);
       const int nc = __popc(km);
       if (keep) cid[__popc(km & lt)] = v;
       __syncwarp();
 
       // ---- a5: bulk distance computation (§VI)
-      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, bar,
-                                                    phase, a.cosine, lane);
+      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, a.cosine,
+                                                    lane);
       n_dist += nc;
       n_exp += 1;
 
@@ -621,6 +753,12 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       {
         uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na > 0 ? A[0] : KEY_MAX);
         uint64_t nxt = umin64(qhead, warp_min_key(key));
+#ifdef SONG_DEBUG
+        if (qi == 0 && lane < 32)
+          printf("it %d lane %d now %llx nc %d cid %d dist %f key %llx qhead %llx nxt %llx q0 %llx\n", iters, lane,
+                 (unsigned long long)now, nc, myid, dist, (unsigned long long)key, (unsigned long long)qhead,
+                 (unsigned long long)nxt, (unsigned long long)q.v[0]);
+#endif
         if (nxt != KEY_MAX && lane < a.degree)
           adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
         else
@@ -628,26 +766,28 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       }
       // visited insert of the selected candidates
       if (BLOOM) {
-        if (sel) bs.insert(myid);
+        bs.insert(myid, sel);
       } else {
-        if (used + ns > ((3 << a.table_log2) >> 2)) {
+        if (used + ns > ((1 << a.table_log2) >> 1)) {
           // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
           for (int i = lane; i < tslots; i += 32) table[i] = EMPTY;
           __syncwarp();
           if (QR > 0) {
 #pragma unroll
             for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
-              if (q.v[r] != KEY_MAX) hs.insert(key_id(q.v[r]));
-              if (tk_r.v[r] != KEY_MAX) hs.insert(key_id(tk_r.v[r]));
+              hs.insert(key_id(q.v[r]), q.v[r] != KEY_MAX);
+              hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
             }
           } else {
-            for (int i = lane; i < na; i += 32) hs.insert(key_id(A[i]));
-            for (int i = lane; i < tsize; i += 32) hs.insert(key_id(tk[i]));
+            for (int i0 = 0; i0 < na; i0 += 32)
+              hs.insert(i0 + lane < na ? key_id(A[i0 + lane]) : 0, i0 + lane < na);
+            for (int i0 = 0; i0 < tsize; i0 += 32)
+              hs.insert(i0 + lane < tsize ? key_id(tk[i0 + lane]) : 0, i0 + lane < tsize);
           }
           used = na + tsize;
           __syncwarp();
         }
-        const bool took = sel ? hs.insert(myid) : false;
+        const bool took = hs.insert(myid, sel);
         used += __popc(__ballot_sync(FULL, took));
       }
       __syncwarp();
@@ -658,30 +798,26 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
         merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
 #pragma unroll
         for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
-          if (r * 32 + lane >= L) {
-            if (!BLOOM && q.v[r] != KEY_MAX) hs.erase(key_id(q.v[r]));
-            q.v[r] = KEY_MAX;
-          }
+          const bool beyond = r * 32 + lane >= L;
+          if (!BLOOM) hs.erase(key_id(q.v[r]), beyond && q.v[r] != KEY_MAX);
+          q.v[r] = beyond ? KEY_MAX : q.v[r];
         }
-        if (!BLOOM && out != KEY_MAX) hs.erase(key_id(out));
+        if (!BLOOM) hs.erase(key_id(out), out != KEY_MAX);
       } else {
         key = bitonic_sort32<false>(key, lane);
         keys32[lane] = key;
         __syncwarp();
-        for (int i = lane; i < na; i += 32) {
-          uint64_t x = A[i];
-          int p = i + count_below(keys32, ns, x);
-          if (p < L)
-            qb[p] = x;
-          else if (!BLOOM)
-            hs.erase(key_id(x));
+        for (int i0 = 0; i0 < na; i0 += 32) {
+          const int i = i0 + lane;
+          const uint64_t x = i < na ? A[i] : KEY_MAX;
+          const int p = i + count_below(keys32, ns, x);
+          if (i < na && p < L) qb[p] = x;
+          if (!BLOOM) hs.erase(key_id(x), i < na && p >= L);
         }
-        if (lane < ns) {
-          int p = lane + count_below(A, na, key);
-          if (p < L)
-            qb[p] = key;
-          else if (!BLOOM)
-            hs.erase(key_id(key));
+        {
+          const int p = lane + count_below(A, na, key);
+          if (lane < ns && p < L) qb[p] = key;
+          if (!BLOOM) hs.erase(key_id(key), lane < ns && p >= L);
         }
         uint64_t* t = qa;
         qa = qb;

@@ -171,8 +171,9 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
     if (s.table_log2 < 5) s.table_log2 = 5;
     tbytes = (1 << s.table_log2) / 8;
   } else {
-    // live keys <= |q| + |topk| + 32 new ones <= 2L + 32; load factor <= 1/2
-    s.table_log2 = next_pow2_log2(2ll * (2 * L + 32));
+    // live keys <= |q| + |topk| + 32 new ones <= 2L + 32; slots >= 4x that, so
+    // live + tombstones stay <= 1/2 of the table (rebuild threshold)
+    s.table_log2 = next_pow2_log2(4ll * (2 * L + 32));
     tbytes = (1 << s.table_log2) * 4;
   }
   s.nch = (dpad + 127) / 128;

@@ -17,7 +17,7 @@ from typing import Optional, Tuple
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libsong.so")
+LIB_PATH = os.environ.get("SONG_LIB", os.path.join(_PKG, "libsong.so"))
 
 L2, IP, COSINE = 0, 1, 2
 METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
