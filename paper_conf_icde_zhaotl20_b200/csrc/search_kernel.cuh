@@ -60,6 +60,7 @@ struct SearchArgs {
   int entry, max_iters, id_offset;
   int cosine;      // MET_DOT: 1 -> 1 - dot, 0 -> -dot
   int dedup;       // 1 if some adjacency row repeats an id
+  int rebuild_at;  // hash: rebuild when live + tombstones would exceed this
   int warp_smem_bytes;
 };
 
@@ -201,13 +202,15 @@ struct HashSet {
   __device__ __forceinline__ bool contains(int v, bool act) const {
     const unsigned mask = (1u << log2) - 1;
     unsigned h = home(v);
-    bool found = false;
+    int s = act ? slot[h] : EMPTY;  // first probe, peeled
+    bool found = act && s == v;
+    act = act && !found && s != EMPTY;
     while (__any_sync(FULL, act)) {
       if (act) {
-        const int s = slot[h];
+        h = (h + 1) & mask;
+        s = slot[h];
         found = (s == v);
         act = !found && s != EMPTY;
-        h = (h + 1) & mask;
       }
     }
     return found;
@@ -237,17 +240,15 @@ struct HashSet {
   __device__ __forceinline__ void erase(int v, bool act) {
     const unsigned mask = (1u << log2) - 1;
     unsigned h = home(v);
+    int s = act ? slot[h] : EMPTY;  // first probe, peeled
+    if (act && s == v) slot[h] = TOMB;
+    act = act && s != v && s != EMPTY;
     while (__any_sync(FULL, act)) {
       if (act) {
-        const int s = slot[h];
-        if (s == v) {
-          slot[h] = TOMB;
-          act = false;
-        } else if (s == EMPTY) {
-          act = false;
-        } else {
-          h = (h + 1) & mask;
-        }
+        h = (h + 1) & mask;
+        s = slot[h];
+        if (s == v) slot[h] = TOMB;
+        act = s != v && s != EMPTY;
       }
     }
   }
@@ -300,10 +301,9 @@ __device__ __forceinline__ uint64_t bitonic_sort32(uint64_t key, int lane) {
   for (int k = 2; k <= 32; k <<= 1) {
 #pragma unroll
     for (int j = k >> 1; j > 0; j >>= 1) {
-      uint64_t other = __shfl_xor_sync(FULL, key, j);
-      bool ascending = ((lane & k) == 0) != DESC;
-      bool lower = (lane & j) == 0;
-      key = (lower == ascending) ? umin64(key, other) : umax64(key, other);
+      const uint64_t other = __shfl_xor_sync(FULL, key, j);
+      const bool take_min = (((lane & j) == 0) == (((lane & k) == 0) != DESC));
+      key = ((other < key) == take_min) ? other : key;  // one 64-bit compare
     }
   }
   return key;
@@ -412,18 +412,21 @@ template <int QR>
 __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int lane, uint64_t& out) {
   // first half-cleaner of the 64*QR-long bitonic sequence [q asc | MAX.. | s desc]
   // only touches the last q register (the MAX block pairs with the rest)
-  const uint64_t lo = umin64(q.v[QR - 1], sdesc);
-  out = umax64(q.v[QR - 1], sdesc);
-  q.v[QR - 1] = lo;
+  {
+    const bool lt = q.v[QR - 1] < sdesc;
+    out = lt ? sdesc : q.v[QR - 1];
+    q.v[QR - 1] = lt ? q.v[QR - 1] : sdesc;
+  }
   // the lower half is bitonic: finish the merge (ascending)
 #pragma unroll
   for (int m = QR / 2; m >= 1; m >>= 1) {
 #pragma unroll
     for (int r = 0; r < QR; ++r) {
       if ((r & m) == 0) {
-        uint64_t a = q.v[r], b = q.v[r + m];
-        q.v[r] = umin64(a, b);
-        q.v[r + m] = umax64(a, b);
+        const uint64_t a = q.v[r], b = q.v[r + m];
+        const bool lt = a < b;
+        q.v[r] = lt ? a : b;
+        q.v[r + m] = lt ? b : a;
       }
     }
   }
@@ -432,8 +435,8 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
     const bool lower = (lane & j) == 0;
 #pragma unroll
     for (int r = 0; r < QR; ++r) {
-      uint64_t o = __shfl_xor_sync(FULL, q.v[r], j);
-      q.v[r] = lower ? umin64(q.v[r], o) : umax64(q.v[r], o);
+      const uint64_t o = __shfl_xor_sync(FULL, q.v[r], j);
+      q.v[r] = ((o < q.v[r]) == lower) ? o : q.v[r];
     }
   }
 }
@@ -445,9 +448,16 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
 // register cost, then each lane reads back only its own 16 B slices (no
 // cross-lane hazard) and a transposed butterfly reduces the R partial sums.
 // Lane j (< nc) receives candidate j's distance.  NCH = 16 B chunks per lane.
+#ifndef SONG_STAGE_ROWS
+#define SONG_STAGE_ROWS 8
+#endif
+#ifndef SONG_STAGE_BUFS
+#define SONG_STAGE_BUFS 1
+#endif
 template <int NCH>
-struct StageRows {
-  static constexpr int R = (NCH >= 8) ? 4 : (32 / NCH);  // rows per round
+struct StageRows {  // rows per round: min(SONG_STAGE_ROWS, 32 / NCH), >= 4
+  static constexpr int R = (NCH >= 8) ? 4 : ((32 / NCH) < SONG_STAGE_ROWS ? (32 / NCH) : SONG_STAGE_ROWS);
+  static constexpr int NBUF = SONG_STAGE_BUFS;  // rounds in flight
 };
 
 __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
@@ -501,11 +511,31 @@ __device__ __forceinline__ uint64_t acc4(uint64_t acc, uint64_t q01, uint64_t q2
   return acc;
 }
 
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// wait until at most n committed groups of this thread are still in flight
+__device__ __forceinline__ void cp_async_wait_pending(int n) {
+  if (n <= 0)
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+  else if (n == 1)
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
+  else if (n == 2)
+    asm volatile("cp.async.wait_group 2;" ::: "memory");
+  else
+    asm volatile("cp.async.wait_group 3;" ::: "memory");
+}
+
+// Rounds of R rows are software-pipelined over NBUF stage buffers: round k+1
+// (and k+2 ...) are in flight while round k is reduced.
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
-                                               float* stage, int cosine, int lane) {
+                                               float* stage, uint64_t* rowp, int cosine,
+                                               int lane) {
   constexpr int R = StageRows<NCH>::R;
+  constexpr int NBUF = StageRows<NCH>::NBUF;
   constexpr int LR = Log2<R>::value;
   constexpr int G = R < 8 ? R : 8;  // rows per uniform compute group
   const int d4 = dpad >> 2;
@@ -516,30 +546,36 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     q01[c] = f2pack(qv[c].x, qv[c].y);
     q23[c] = f2pack(qv[c].z, qv[c].w);
   }
-  for (int b = 0; b < nc; b += R) {
-    const int rows = min(R, nc - b);
-    // ---- issue: every row of the round in flight at once
+  // lane j resolves candidate j's row address once
+  if (lane < nc) rowp[lane] = reinterpret_cast<uint64_t>(data + (int64_t)cid[lane] * dpad);
+  __syncwarp();
+  const int rounds = (nc + R - 1) / R;
+  // issue round k: one LDGSTS per row per 16 B chunk, into buffer k % NBUF
+  auto issue = [&](int k) {
+    float4* dst = reinterpret_cast<float4*>(stage + (size_t)(k % NBUF) * R * dpad) + lane;
+    const int r1 = min(nc, (k + 1) * R);
+    for (int r = k * R; r < r1; ++r, dst += d4) {
+      const float4* src = reinterpret_cast<const float4*>(rowp[r]) + lane;
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (r < rows) {
-        const float4* src = reinterpret_cast<const float4*>(data + (int64_t)cid[b + r] * dpad);
-        float4* dst = reinterpret_cast<float4*>(stage + (size_t)r * dpad);
-#pragma unroll
-        for (int c = 0; c < NCH; ++c) {
-          const int idx = c * 32 + lane;
-          if (idx < d4) cp_async16(dst + idx, src + idx);
-        }
-      }
+      for (int c = 0; c < NCH; ++c)
+        if (c * 32 + lane < d4) cp_async16(dst + c * 32, src + c * 32);
     }
-    cp_async_wait_all();
+    cp_async_commit();
+  };
+  for (int k = 0; k < NBUF && k < rounds; ++k) issue(k);
+  for (int k = 0; k < rounds; ++k) {
+    const int b = k * R;
+    const int rows = min(R, nc - b);
+    cp_async_wait_pending(min(NBUF - 1, rounds - 1 - k));
     // ---- compute: lane owns its 16 B slices of every staged row
+    const float* buf = stage + (size_t)(k % NBUF) * R * dpad;
     float part[R];
 #pragma unroll
     for (int g = 0; g < R; g += G) {
       if (g < rows) {
 #pragma unroll
         for (int r = g; r < g + G; ++r) {
-          const float4* row = reinterpret_cast<const float4*>(stage + (size_t)r * dpad);
+          const float4* row = reinterpret_cast<const float4*>(buf + (size_t)r * dpad);
           uint64_t acc = 0;
 #pragma unroll
           for (int c = 0; c < NCH; ++c) {
@@ -553,19 +589,10 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
         for (int r = g; r < g + G; ++r) part[r] = 0.0f;
       }
     }
-#ifdef SONG_DEBUG
-    if (lane < 2) {
-      for (int r = 0; r < rows; ++r) {
-        const float4 x = reinterpret_cast<const float4*>(stage + (size_t)r * dpad)[lane];
-        printf("bd lane %d row %d id %d x %f %f %f %f q %f part %f\n", lane, r, cid[b + r], x.x, x.y, x.z, x.w, qv[0].x, part[r]);
-      }
-    }
-#endif
-    float tot = transpose_reduce<R>(part, lane);
-#ifdef SONG_DEBUG
-    if (lane < 4) printf("bd lane %d tot %f\n", lane, tot);
-#endif
-    float got = __shfl_sync(FULL, tot, ((lane - b) & (R - 1)) << (5 - LR));
+    // buffer k % NBUF is free again (this lane read only its own slices)
+    if (k + NBUF < rounds) issue(k + NBUF);
+    const float tot = transpose_reduce<R>(part, lane);
+    const float got = __shfl_sync(FULL, tot, ((lane - b) & (R - 1)) << (5 - LR));
     if (lane >= b && lane < b + R) mine = got;
   }
   if (METRIC == MET_DOT) mine = cosine ? 1.0f - mine : -mine;  // 1 - cos / -<q,x>
@@ -583,9 +610,10 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
   float* stage = reinterpret_cast<float*>(base);                       // R rows
-  int* cid = reinterpret_cast<int*>(base + (size_t)R * a.dpad * 4 + 16);  // 32 ids
+  int* cid = reinterpret_cast<int*>(base + (size_t)StageRows<NCH>::NBUF * R * a.dpad * 4 + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
-  uint64_t* qa = keys32 + 32;                                           // QR == 0 only
+  uint64_t* rowp = keys32 + 32;                                         // 32 row pointers
+  uint64_t* qa = rowp + 32;                                             // QR == 0 only
   uint64_t* qb = qa + (QR == 0 ? L : 0);
   uint64_t* tk = qb + (QR == 0 ? L : 0);
   int* table = reinterpret_cast<int*>(tk + (QR == 0 ? L : 0));
@@ -650,7 +678,8 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
     for (int i = lane; i < tslots; i += 32) table[i] = BLOOM ? 0 : EMPTY;
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, a.cosine, lane);
+    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, rowp, a.cosine,
+                                                lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     if (BLOOM)
       bs.insert(a.entry, lane == 0);
@@ -737,8 +766,8 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       __syncwarp();
 
       // ---- a5: bulk distance computation (§VI)
-      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, a.cosine,
-                                                    lane);
+      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, rowp,
+                                                    a.cosine, lane);
       n_dist += nc;
       n_exp += 1;
 
@@ -768,7 +797,7 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
       if (BLOOM) {
         bs.insert(myid, sel);
       } else {
-        if (used + ns > ((1 << a.table_log2) >> 1)) {
+        if (used + ns > a.rebuild_at) {
           // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
           for (int i = lane; i < tslots; i += 32) table[i] = EMPTY;
           __syncwarp();
@@ -849,7 +878,7 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
           dists_o[i] = __int_as_float(0x7f800000);
         }
       }
-      qa = keys32 + 32;
+      qa = rowp + 32;
       qb = qa + L;
     }
     if (a.counters_out && lane == 0) {

@@ -155,9 +155,16 @@ int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* a
   return SONG_OK;
 }
 
+#ifndef SONG_HASH_FACTOR
+#define SONG_HASH_FACTOR 8
+#endif
+#ifndef SONG_HASH_REBUILD_NUM  // rebuild at NUM/16 occupancy
+#define SONG_HASH_REBUILD_NUM 4
+#endif
 // per-warp shared memory of the search kernel
 struct Shape {
   int table_log2;
+  int rebuild_at;
   int warp_bytes;
   int qr;  // register queue width (L <= 32*qr), 0 = shared-memory queues
   int nch;
@@ -166,21 +173,27 @@ struct Shape {
 Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   Shape s;
   int tbytes;
+  s.rebuild_at = 0;
   if (bloom) {
     s.table_log2 = bloom_log2_bits > 0 ? bloom_log2_bits : next_pow2_log2(80ll * L);
     if (s.table_log2 < 5) s.table_log2 = 5;
     tbytes = (1 << s.table_log2) / 8;
   } else {
-    // live keys <= |q| + |topk| + 32 new ones <= 2L + 32; slots >= 4x that, so
-    // live + tombstones stay <= 1/2 of the table (rebuild threshold)
-    s.table_log2 = next_pow2_log2(4ll * (2 * L + 32));
+    // live keys <= |q| + |topk| + 32 new ones <= 2L + 32.  Register-queue
+    // sizes get >= 8x that many slots and rebuild at 1/4 occupancy (about one
+    // probe per operation); shared-memory queues (L > 128) get >= 2x and
+    // rebuild at 3/4 to bound shared memory.
+    const bool big = L > 128;
+    s.table_log2 = next_pow2_log2((big ? 2ll : (long long)SONG_HASH_FACTOR) * (2 * L + 32));
+    s.rebuild_at = big ? (3 << s.table_log2) / 4 : (SONG_HASH_REBUILD_NUM << s.table_log2) / 16;
     tbytes = (1 << s.table_log2) * 4;
   }
   s.nch = (dpad + 127) / 128;
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
-  const int rows = s.nch >= 8 ? 4 : 32 / s.nch;  // StageRows<NCH>::R
+  const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
-  s.warp_bytes = rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 : 0) + tbytes;
+  s.warp_bytes = SONG_STAGE_BUFS * rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 : 0) +
+                 tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;
 }
@@ -263,6 +276,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   const bool bloom = p->visited == SONG_VISITED_BLOOM;
   Shape sh = search_shape(p->queue_len, bloom, p->bloom_log2_bits, ix->dpad);
   a.table_log2 = sh.table_log2;
+  a.rebuild_at = sh.rebuild_at;
   a.warp_smem_bytes = sh.warp_bytes;
   a.entry = p->entry;
   a.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);
