@@ -74,7 +74,7 @@ typedef struct song_search_params {
   int32_t entry;           /* starting vertex id, 0 <= entry < n */
   int32_t max_iters;       /* expansion cap per query (0 = 1<<30); a query that
                               reaches it is flagged, see song_search_ex */
-  int32_t warps_per_block; /* launch shape: 0 = library default */
+  int32_t warps_per_block; /* launch shape: 0 = library default (4); at most 4 */
   int32_t blocks_per_sm;   /* launch shape: 0 = as many as fit */
   int32_t id_offset;       /* added to every returned id (dataset sharding, P:471:
                               shard-local ids become global ids); default 0 */
@@ -134,8 +134,9 @@ int song_search(song_index* idx, const float* queries, int64_t nq, int32_t K,
 /* Search with DEVICE buffers on a caller stream; asynchronous (returns after
  * enqueueing).  counters_out, if not NULL, receives [nq][2] int32
  * (distance computations, expansions) per query — the algorithmic work that
- * defines the roofline bytes.  A query that hits max_iters or has a
- * non-finite value gets ids -1; song_index_last_status() reports it.
+ * defines the roofline bytes.  A query with a non-finite value gets ids -1;
+ * one that reaches max_iters returns its partial topk; both are reported by
+ * song_index_last_status().
  * Errors detectable before launch: SONG_EINVAL, SONG_EUNSUPPORTED, SONG_ECUDA. */
 int song_search_ex(song_index* idx, const song_search_params* params,
                    const float* queries, int64_t nq, int32_t* ids_out, float* dists_out,

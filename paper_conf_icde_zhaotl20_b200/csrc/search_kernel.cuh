@@ -140,97 +140,57 @@ __device__ __forceinline__ void fence_proxy_async() {
 }
 
 // ---------------------------------------------------------------- visited --
-// Open-addressing hash in shared memory, linear probing.  Every lane
-// runs its own probe sequence, so up to 32 operations proceed in parallel;
-// all loops are warp-collective (trip count decided by __any_sync) so the
-// warp stays converged for the shuffles that follow.
-#ifdef SONG_OLD_HASH
+// Open-addressing hash in shared memory organised as buckets of four
+// 4-byte slots: one LDS.128 reads a whole bucket, so at the table's low load
+// (<= 1/4) almost every operation resolves with a single probe; buckets are
+// probed linearly (open addressing).  Every lane runs its own probe sequence,
+// so up to 32 operations proceed in parallel, and all loops are
+// warp-collective (trip count decided by __any_sync) so the warp stays
+// converged for the shuffles that follow.
 struct HashSet {
   int* slot;
-  int log2;
+  int log2;  // slots = 2^log2, buckets = 2^(log2 - 2)
   __device__ __forceinline__ unsigned home(int v) const {
-    return ((uint32_t)v * 0x9E3779B1u) >> (32 - log2);
+    return ((uint32_t)v * 0x9E3779B1u) >> (34 - log2);
   }
-  __device__ __forceinline__ bool contains(int v, bool act) const {
-    if (!act) return false;
-    unsigned mask = (1u << log2) - 1, h = home(v);
-    while (true) {
-      int s = slot[h];
-      if (s == v) return true;
-      if (s == EMPTY) return false;
-      h = (h + 1) & mask;
-    }
-  }
-  __device__ __forceinline__ bool insert(int v, bool act) {
-    bool r = false;
-    if (act) {
-    unsigned mask = (1u << log2) - 1, h = home(v);
-    while (true) {
-      int s = slot[h];
-      if (s == EMPTY || s == TOMB) {
-        int old = atomicCAS(&slot[h], s, v);
-        if (old == s) { r = (s == EMPTY); break; }
-        continue;
-      }
-      h = (h + 1) & mask;
-    }
-    }
-    __syncwarp();
-    return r;
-  }
-  __device__ __forceinline__ void erase(int v, bool act) {
-    if (act) {
-    unsigned mask = (1u << log2) - 1, h = home(v);
-    while (true) {
-      int s = slot[h];
-      if (s == v) { slot[h] = TOMB; break; }
-      if (s == EMPTY) break;
-      h = (h + 1) & mask;
-    }
-    }
-    __syncwarp();
-  }
-};
-#else
-struct HashSet {
-  int* slot;
-  int log2;
-  __device__ __forceinline__ unsigned home(int v) const {
-    return ((uint32_t)v * 0x9E3779B1u) >> (32 - log2);
+  __device__ __forceinline__ int4 bucket(unsigned b) const {
+    return reinterpret_cast<const int4*>(slot)[b];
   }
   // membership of v for lanes with act; result false elsewhere
   __device__ __forceinline__ bool contains(int v, bool act) const {
-    const unsigned mask = (1u << log2) - 1;
-    unsigned h = home(v);
-    int s = act ? slot[h] : EMPTY;  // first probe, peeled
-    bool found = act && s == v;
-    act = act && !found && s != EMPTY;
+    const unsigned mask = (1u << (log2 - 2)) - 1;
+    unsigned b = home(v);
+    bool found = false;
     while (__any_sync(FULL, act)) {
       if (act) {
-        h = (h + 1) & mask;
-        s = slot[h];
-        found = (s == v);
-        act = !found && s != EMPTY;
+        const int4 s = bucket(b);
+        found = (s.x == v) | (s.y == v) | (s.z == v) | (s.w == v);
+        const bool open = (s.x == EMPTY) | (s.y == EMPTY) | (s.z == EMPTY) | (s.w == EMPTY);
+        act = !found && !open;
+        b = (b + 1) & mask;
       }
     }
     return found;
   }
   // insert v (not present) for lanes with act; true when an EMPTY slot was used
   __device__ __forceinline__ bool insert(int v, bool act) {
-    const unsigned mask = (1u << log2) - 1;
-    unsigned h = home(v);
+    const unsigned mask = (1u << (log2 - 2)) - 1;
+    unsigned b = home(v);
     bool took_empty = false;
     while (__any_sync(FULL, act)) {
       if (act) {
-        const int s = slot[h];
-        if (s == EMPTY || s == TOMB) {
-          const int old = atomicCAS(&slot[h], s, v);
-          if (old == s) {
+        const int4 s = bucket(b);
+        const bool f0 = s.x < 0, f1 = s.y < 0, f2 = s.z < 0, f3 = s.w < 0;  // EMPTY or TOMB
+        if (f0 | f1 | f2 | f3) {
+          const int j = f0 ? 0 : f1 ? 1 : f2 ? 2 : 3;
+          const int old_v = f0 ? s.x : f1 ? s.y : f2 ? s.z : s.w;
+          const int old = atomicCAS(&slot[4 * b + j], old_v, v);
+          if (old == old_v) {
             act = false;
-            took_empty = (s == EMPTY);
-          }  // else: lost the race for this slot, re-read it
+            took_empty = (old_v == EMPTY);
+          }  // else: lost the race for this slot, re-read the bucket
         } else {
-          h = (h + 1) & mask;
+          b = (b + 1) & mask;
         }
       }
     }
@@ -238,22 +198,23 @@ struct HashSet {
   }
   // delete v (present) for lanes with act (§IV-E): the slot becomes a tombstone
   __device__ __forceinline__ void erase(int v, bool act) {
-    const unsigned mask = (1u << log2) - 1;
-    unsigned h = home(v);
-    int s = act ? slot[h] : EMPTY;  // first probe, peeled
-    if (act && s == v) slot[h] = TOMB;
-    act = act && s != v && s != EMPTY;
+    const unsigned mask = (1u << (log2 - 2)) - 1;
+    unsigned b = home(v);
     while (__any_sync(FULL, act)) {
       if (act) {
-        h = (h + 1) & mask;
-        s = slot[h];
-        if (s == v) slot[h] = TOMB;
-        act = s != v && s != EMPTY;
+        const int4 s = bucket(b);
+        const bool h0 = s.x == v, h1 = s.y == v, h2 = s.z == v, h3 = s.w == v;
+        if (h0 | h1 | h2 | h3) {
+          slot[4 * b + (h0 ? 0 : h1 ? 1 : h2 ? 2 : 3)] = TOMB;
+          act = false;
+        } else {
+          act = !((s.x == EMPTY) | (s.y == EMPTY) | (s.z == EMPTY) | (s.w == EMPTY));
+          b = (b + 1) & mask;
+        }
       }
     }
   }
 };
-#endif
 
 // Bloom filter with the k = 7 double-hashing spec of reading A8:
 // bit_i = (h1 + i*h2) mod m, h1 = fmix32(id), h2 = fmix32(id ^ 0x5bd1e995) | 1.
@@ -465,6 +426,15 @@ __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
                : "memory");
 }
 
+// predicated form: no branch around the copy
+__device__ __forceinline__ void cp_async16_if(bool p, uint32_t dst, const void* src) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t"
+      "@q cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(dst),
+      "l"(src), "r"((int)p)
+      : "memory");
+}
+
 __device__ __forceinline__ void cp_async_wait_all() {
   asm volatile("cp.async.wait_all;" ::: "memory");
 }
@@ -551,14 +521,18 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
   __syncwarp();
   const int rounds = (nc + R - 1) / R;
   // issue round k: one LDGSTS per row per 16 B chunk, into buffer k % NBUF
+  const uint32_t stage_s = smem_u32(stage) + 16u * lane;
+  const uint32_t rowbytes = 4u * (uint32_t)dpad;
   auto issue = [&](int k) {
-    float4* dst = reinterpret_cast<float4*>(stage + (size_t)(k % NBUF) * R * dpad) + lane;
-    const int r1 = min(nc, (k + 1) * R);
-    for (int r = k * R; r < r1; ++r, dst += d4) {
-      const float4* src = reinterpret_cast<const float4*>(rowp[r]) + lane;
+    const uint32_t dst0 = stage_s + (uint32_t)((k % NBUF) * R) * rowbytes;
+    const int rows = min(R, nc - k * R);
+#pragma unroll
+    for (int rr = 0; rr < R; ++rr) {
+      const bool on = rr < rows;
+      const float4* src = reinterpret_cast<const float4*>(rowp[on ? k * R + rr : 0]) + lane;
 #pragma unroll
       for (int c = 0; c < NCH; ++c)
-        if (c * 32 + lane < d4) cp_async16(dst + c * 32, src + c * 32);
+        cp_async16_if(on && (c * 32 + lane < d4), dst0 + rr * rowbytes + 512u * c, src + c * 32);
     }
     cp_async_commit();
   };
@@ -573,15 +547,13 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
 #pragma unroll
     for (int g = 0; g < R; g += G) {
       if (g < rows) {
+        const float4* row = reinterpret_cast<const float4*>(buf) + (size_t)g * d4 + lane;
 #pragma unroll
-        for (int r = g; r < g + G; ++r) {
-          const float4* row = reinterpret_cast<const float4*>(buf + (size_t)r * dpad);
+        for (int r = g; r < g + G; ++r, row += d4) {
           uint64_t acc = 0;
 #pragma unroll
-          for (int c = 0; c < NCH; ++c) {
-            const int idx = c * 32 + lane;
-            if (idx < d4) acc = acc4<METRIC>(acc, q01[c], q23[c], row[idx]);
-          }
+          for (int c = 0; c < NCH; ++c)
+            if (c * 32 + lane < d4) acc = acc4<METRIC>(acc, q01[c], q23[c], row[c * 32]);
           part[r] = f2sum(acc);
         }
       } else {
@@ -600,9 +572,15 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
 }
 
 // ---------------------------------------------------------- the kernel --
+#ifndef SONG_LB_THREADS
+#define SONG_LB_THREADS 128
+#endif
+#ifndef SONG_LB_BLOCKS
+#define SONG_LB_BLOCKS 6
+#endif
 // QR > 0: q / topk in registers (queue_len <= 32*QR); QR == 0: shared memory.
 template <int NCH, int METRIC, bool BLOOM, int QR>
-__global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
+__global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH>::R;
   const int lane = threadIdx.x & 31;
@@ -616,7 +594,8 @@ __global__ void __launch_bounds__(256) song_search_kernel(const SearchArgs a) {
   uint64_t* qa = rowp + 32;                                             // QR == 0 only
   uint64_t* qb = qa + (QR == 0 ? L : 0);
   uint64_t* tk = qb + (QR == 0 ? L : 0);
-  int* table = reinterpret_cast<int*>(tk + (QR == 0 ? L : 0));
+  int* table = reinterpret_cast<int*>(                                  // 16 B aligned
+      (reinterpret_cast<uintptr_t>(tk + (QR == 0 ? L : 0)) + 15) & ~uintptr_t(15));
   const int tslots = BLOOM ? ((1 << a.table_log2) >> 5) : (1 << a.table_log2);
   HashSet hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};

@@ -192,7 +192,7 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
   const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
-  s.warp_bytes = SONG_STAGE_BUFS * rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 : 0) +
+  s.warp_bytes = SONG_STAGE_BUFS * rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;
@@ -246,8 +246,8 @@ int check_params(const song_index* ix, const song_search_params* p) {
   if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
   if (p->bloom_log2_bits < 0 || p->bloom_log2_bits > 24)
     return fail(SONG_EUNSUPPORTED, "bloom_log2_bits %d outside [0, 24]", p->bloom_log2_bits);
-  if (p->warps_per_block < 0 || p->warps_per_block > 8)
-    return fail(SONG_EINVAL, "warps_per_block %d outside [0, 8]", p->warps_per_block);
+  if (p->warps_per_block < 0 || p->warps_per_block > SONG_LB_THREADS / 32)
+    return fail(SONG_EINVAL, "warps_per_block %d outside [0, %d]", p->warps_per_block, SONG_LB_THREADS / 32);
   if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
   if (p->reserved != 0) return fail(SONG_EINVAL, "reserved must be 0");
   return SONG_OK;

@@ -110,7 +110,7 @@ def sift100k():
 
 
 @pytest.mark.parametrize("L,visited,warps", [(10, "hash", 4), (16, "hash", 1), (64, "hash", 4),
-                                            (200, "hash", 8), (64, "bloom", 4),
+                                            (200, "hash", 3), (64, "bloom", 4),
                                             (1024, "hash", 2)])
 def test_sift_integer_bit_exact(sift100k, L, visited, warps):
     cfg, x, q, adj = sift100k
