@@ -260,3 +260,29 @@ def test_merge_topk_matches_plain_merge():
     ei, ed = oracle.merge_shards(list(ids), list(dists), K)
     np.testing.assert_array_equal(oi.cpu().numpy(), ei)
     np.testing.assert_array_equal(od.cpu().numpy(), ed)
+
+
+def test_dataset_sharding_emulated_on_one_gpu(sift100k):
+    """P:471 on one GPU: G shards searched one after another with global ids
+    (id_offset), merged by song_merge_topk; bit-exact vs the oracle per shard +
+    the plain merge (SURVEY §4 single-GPU emulation)."""
+    from paper_conf_icde_zhaotl20_b200 import sharded
+    cfg, x, q, adj = sift100k
+    s = song()
+    G, K, L = 3, 10, 40
+    gi, gd, per_i, per_d = [], [], [], []
+    for lo, hi in sharded.shard_ranges(x.shape[0], G):
+        xs = x[lo:hi].contiguous()
+        a = build_graph(xs, degree=32)
+        idx = s.SongIndex(xs, a)
+        i, d = idx.search(q, params=s.Params(K=K, queue_len=L, id_offset=lo))
+        gi.append(i)
+        gd.append(d)
+        oi, od, _, _ = oracle.search(xs.cpu().numpy(), a.cpu().numpy(), q.cpu().numpy(), K, L,
+                                     nthreads=8)
+        per_i.append(np.where(oi >= 0, oi + lo, -1))
+        per_d.append(od)
+    mi, md = s.merge_topk(torch.stack(gi), torch.stack(gd), K)
+    ei, ed = oracle.merge_shards(per_i, per_d, K)
+    np.testing.assert_array_equal(mi.cpu().numpy(), ei)
+    np.testing.assert_array_equal(md.cpu().numpy(), ed)

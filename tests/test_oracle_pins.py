@@ -239,3 +239,15 @@ def test_recall_definition():
     """Recall(A) = |A ∩ B| / |B|, averaged over queries."""
     assert oracle.recall([[1, 2, 3]], [[3, 4, 5]]) == pytest.approx(1 / 3)
     assert oracle.recall([[1, 2], [5, 6]], [[1, 2], [7, 8]]) == pytest.approx(0.5)
+
+
+def test_merge_shards_definition():
+    """P:471 "merge the results": K smallest (dist, id) over all shards, ties
+    by id, padding (-1, inf) ignored; worked by hand."""
+    ids = [np.array([[5, 9, -1]]), np.array([[2, 7, 8]])]
+    d = [np.array([[1.0, 3.0, np.inf]], np.float32), np.array([[1.0, 2.0, 9.0]], np.float32)]
+    i, dd = oracle.merge_shards(ids, d, 4)
+    assert i.tolist() == [[2, 5, 7, 9]]
+    assert dd.tolist() == [[1.0, 1.0, 2.0, 3.0]]
+    i, dd = oracle.merge_shards([np.array([[-1, -1]])], [np.full((1, 2), np.inf, np.float32)], 2)
+    assert i.tolist() == [[-1, -1]] and np.isinf(dd).all()
