@@ -286,3 +286,29 @@ def test_dataset_sharding_emulated_on_one_gpu(sift100k):
     ei, ed = oracle.merge_shards(per_i, per_d, K)
     np.testing.assert_array_equal(mi.cpu().numpy(), ei)
     np.testing.assert_array_equal(md.cpu().numpy(), ed)
+
+
+@pytest.mark.slow
+def test_sift1m_full_size_sampled_parity():
+    """BASELINE configs[1] at full size (1M x 128, degree 32, 10,000 queries) in
+    bench.py's launch configuration (default launch shape, queue_len 48 = the
+    recall@10 >= 0.95 operating point): the oracle recomputes a sample of 300
+    queries one by one; ids, distances and counters must be bit-exact."""
+    cfg = CONFIGS["sift1m"]
+    x, q = make_data(cfg, device="cuda")
+    adj = build_graph(x, degree=cfg.degree)
+    s = song()
+    idx = s.SongIndex(x, adj)
+    ids, d, c = idx.search(q, params=s.Params(K=cfg.K, queue_len=48), counters=True)
+    torch.cuda.synchronize()
+    idx.last_status()
+    rng = np.random.default_rng(0)
+    pick = np.sort(rng.choice(cfg.nq, 300, replace=False))
+    xn, an = x.cpu().numpy(), adj.cpu().numpy()
+    o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 48, nthreads=8)
+    assert_exact((ids.cpu().numpy()[pick], d.cpu().numpy()[pick], c.cpu().numpy()[pick]), o)
+    # properties that hold for every query at any size: sorted, unique, valid ids
+    ii, dd = ids.cpu().numpy(), d.cpu().numpy()
+    assert (np.diff(dd, axis=1) >= 0).all()
+    assert ((ii >= 0) & (ii < cfg.n)).all()
+    assert all(len(set(r)) == cfg.K for r in ii)
