@@ -8,29 +8,30 @@
 //   locate (§V)    the adjacency row of the head (prefetched into registers
 //                  during the previous iteration's maintenance) is filtered:
 //                  padding, repeats (match.any, only if the index has them)
-//                  and visited ids (32 parallel hash probes), compacted by a
-//                  ballot
-//   distance (§VI) every surviving candidate lane issues ONE bulk copy
-//                  (cp.async.bulk, the TMA engine) of its d*4-byte row into a
-//                  per-warp shared-memory stage, completion on an mbarrier:
-//                  all rows of the iteration are in flight at once with no
-//                  register cost.  Lanes then read 16 B slices (LDS.128,
-//                  conflict-free) and a transposed butterfly reduces R rows in
-//                  R-1+(5-log2 R) shuffles (P:455's shfl_down reduction,
-//                  batched)
-//   maintain (§IV) selected insertion (§IV-D) against topk's max, warp bitonic
-//                  sort of the <= 32 survivors, visited insert, bitonic merge
-//                  into the bounded q (§IV-C) with visited deletion of the
-//                  evicted keys (§IV-E).  For queue_len <= 128 q and topk live
-//                  in registers (sorted, striped over the lanes); larger
-//                  queues use shared-memory arrays and merge-path ranks.
+//                  and visited ids (32 parallel probes of a bucketed hash),
+//                  compacted by a ballot
+//   distance (§VI) rounds of 8 candidate rows: lane j resolves candidate j's
+//                  row address, every row of the round is put in flight at
+//                  once with cp.async (LDGSTS, 16 B per lane per row) into a
+//                  per-warp shared-memory stage — no register cost — then each
+//                  lane reduces its own 16 B slices with packed FFMA2/FADD2 and
+//                  a transposed butterfly sums 8 rows in 9 shuffles (P:455's
+//                  shfl_down reduction, batched)
+//   maintain (§IV) selected insertion (§IV-D) against topk's max, compaction +
+//                  bitonic sort of only the selected keys, visited insert,
+//                  bitonic merge into the bounded q (§IV-C) with visited
+//                  deletion of the evicted keys (§IV-E).  For queue_len <= 128
+//                  q and topk live in registers (sorted, striped over the
+//                  lanes); larger queues use shared-memory arrays and
+//                  merge-path ranks.
 //
 // Priority-queue keys are u64 (orderable(dist) << 32 | id): the (dist, id)
 // total order of DESIGN.md reading A3 as a single integer compare.
 #pragma once
 
-#include <cstdint>
 #include <cuda_runtime.h>
+
+#include <cstdint>
 
 namespace song {
 
@@ -100,43 +101,9 @@ __device__ __forceinline__ uint64_t warp_min_key(uint64_t k) {
   return ((uint64_t)mh << 32) | ml;
 }
 
-// ------------------------------------------------------- async row copies --
+// ------------------------------------------------------- shared addresses --
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
-               "r"(bytes)
-               : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n"
-      "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-
-// one bulk copy (TMA engine) of `bytes` from global to shared, completing on bar
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
-
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
 // ---------------------------------------------------------------- visited --
@@ -268,6 +235,32 @@ __device__ __forceinline__ uint64_t bitonic_sort32(uint64_t key, int lane) {
     }
   }
   return key;
+}
+
+// ascending bitonic sort of each W-lane block (W <= 32, a power of two)
+template <int W>
+__device__ __forceinline__ uint64_t bitonic_sort_w(uint64_t key, int lane) {
+#pragma unroll
+  for (int k = 2; k <= W; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      const uint64_t other = __shfl_xor_sync(FULL, key, j);
+      const bool take_min = (((lane & j) == 0) == ((lane & k) == 0));
+      key = ((other < key) == take_min) ? other : key;
+    }
+  }
+  return key;
+}
+
+// ascending sort of the n (warp-uniform) keys held by lanes [0, n); lanes >= n
+// hold KEY_MAX.  Only the network for the next power of two >= n is run.
+__device__ __forceinline__ uint64_t sort_prefix(uint64_t key, int n, int lane) {
+  if (n <= 1) return key;
+  if (n <= 2) return bitonic_sort_w<2>(key, lane);
+  if (n <= 4) return bitonic_sort_w<4>(key, lane);
+  if (n <= 8) return bitonic_sort_w<8>(key, lane);
+  if (n <= 16) return bitonic_sort_w<16>(key, lane);
+  return bitonic_sort_w<32>(key, lane);
 }
 
 // number of elements of sorted a[0..n) strictly below x
@@ -587,8 +580,9 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   const int warp = threadIdx.x >> 5;
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
-  float* stage = reinterpret_cast<float*>(base);                       // R rows
-  int* cid = reinterpret_cast<int*>(base + (size_t)StageRows<NCH>::NBUF * R * a.dpad * 4 + 16);
+  float* stage = reinterpret_cast<float*>(base);                       // staged rows
+  const size_t stage_bytes = (size_t)StageRows<NCH>::NBUF * R * a.dpad * 4;
+  int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
   uint64_t* rowp = keys32 + 32;                                         // 32 row pointers
   uint64_t* qa = rowp + 32;                                             // QR == 0 only
@@ -755,7 +749,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
       const uint64_t thr = (tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
       const bool sel = (lane < nc) && key < thr;  // selected insertion
-      const int ns = __popc(__ballot_sync(FULL, sel));
+      const unsigned smask = __ballot_sync(FULL, sel);
+      const int ns = __popc(smask);
       if (!sel) key = KEY_MAX;
       // prefetch the adjacency row of the next head = min(q head, best new key)
       {
@@ -772,12 +767,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
         else
           adjv = -1;
       }
-      // visited insert of the selected candidates
-      if (BLOOM) {
-        bs.insert(myid, sel);
-      } else {
+      // visited insert of the selected candidates (hash: rebuild first when
+      // tombstones accumulated — visited = ids(q) ∪ ids(topk))
+      auto visit_selected = [&]() {
+        if (BLOOM) {
+          bs.insert(myid, sel);
+          return;
+        }
         if (used + ns > a.rebuild_at) {
-          // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
           for (int i = lane; i < tslots; i += 32) table[i] = EMPTY;
           __syncwarp();
           if (QR > 0) {
@@ -797,21 +794,30 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
         }
         const bool took = hs.insert(myid, sel);
         used += __popc(__ballot_sync(FULL, took));
-      }
-      __syncwarp();
+      };
       if (QR > 0) {
-        // merge the selected keys into q; evict beyond L (§IV-C) and delete (§IV-E)
-        const uint64_t sdesc = bitonic_sort32<true>(key, lane);
-        uint64_t out;
-        merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
+        if (ns > 0) {  // (ns == 0: q only lost its head, nothing to insert/evict)
+          visit_selected();
+          // compact the selected keys to lanes [0, ns), sort only those
+          if (sel) keys32[__popc(smask & lt)] = key;
+          __syncwarp();
+          uint64_t k2 = lane < ns ? keys32[lane] : KEY_MAX;
+          k2 = sort_prefix(k2, ns, lane);
+          const uint64_t sdesc = __shfl_sync(FULL, k2, 31 - lane);  // descending
+          // merge into q; evict beyond L (§IV-C) and delete from visited (§IV-E)
+          uint64_t out;
+          merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
 #pragma unroll
-        for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
-          const bool beyond = r * 32 + lane >= L;
-          if (!BLOOM) hs.erase(key_id(q.v[r]), beyond && q.v[r] != KEY_MAX);
-          q.v[r] = beyond ? KEY_MAX : q.v[r];
+          for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+            const bool beyond = r * 32 + lane >= L;
+            if (!BLOOM) hs.erase(key_id(q.v[r]), beyond && q.v[r] != KEY_MAX);
+            q.v[r] = beyond ? KEY_MAX : q.v[r];
+          }
+          if (!BLOOM) hs.erase(key_id(out), out != KEY_MAX);
         }
-        if (!BLOOM) hs.erase(key_id(out), out != KEY_MAX);
       } else {
+        visit_selected();
+        __syncwarp();
         key = bitonic_sort32<false>(key, lane);
         keys32[lane] = key;
         __syncwarp();

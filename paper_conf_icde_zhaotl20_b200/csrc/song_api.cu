@@ -192,7 +192,8 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
   const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
-  s.warp_bytes = SONG_STAGE_BUFS * rows * dpad * 4 + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
+  const int stage_bytes = SONG_STAGE_BUFS * rows * dpad * 4;
+  s.warp_bytes = stage_bytes + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;
@@ -217,7 +218,8 @@ int launch_t(const song::SearchArgs& a, int warps, int blocks_per_sm, int num_sm
 }
 
 template <int NCH, int METRIC, bool BLOOM>
-int launch_q(const song::SearchArgs& a, int qr, int warps, int bps, int sms, cudaStream_t st) {
+int launch_q(const song::SearchArgs& a, int qr, int warps, int bps, int sms,
+             cudaStream_t st) {
   switch (qr) {
     case 1: return launch_t<NCH, METRIC, BLOOM, 1>(a, warps, bps, sms, st);
     case 2: return launch_t<NCH, METRIC, BLOOM, 2>(a, warps, bps, sms, st);
@@ -227,8 +229,8 @@ int launch_q(const song::SearchArgs& a, int qr, int warps, int bps, int sms, cud
 }
 
 template <int NCH>
-int launch_m(const song::SearchArgs& a, int metric, bool bloom, int qr, int warps, int bps,
-             int sms, cudaStream_t st) {
+int launch_m(const song::SearchArgs& a, int metric, bool bloom, int qr,
+             int warps, int bps, int sms, cudaStream_t st) {
   if (metric == SONG_L2)
     return bloom ? launch_q<NCH, song::MET_L2, true>(a, qr, warps, bps, sms, st)
                  : launch_q<NCH, song::MET_L2, false>(a, qr, warps, bps, sms, st);
