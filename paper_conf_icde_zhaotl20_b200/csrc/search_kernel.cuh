@@ -491,41 +491,51 @@ __device__ __forceinline__ void cp_async_wait_pending(int n) {
 }
 
 // Rounds of R rows are software-pipelined over NBUF stage buffers: round k+1
-// (and k+2 ...) are in flight while round k is reduced.
+// (and k+2 ...) are in flight while round k is reduced.  Staged rows have a
+// compile-time stride of 128*NCH floats (512*NCH bytes) so every shared-memory
+// address is an immediate offset; lane j holds candidate j's row pointer and
+// rows are broadcast with SHFL (an LDS-sourced address makes ptxas pad every
+// LDGSTS with three dummy LDS).
+template <int NCH>
+struct Stage {
+  static constexpr int STRIDE = 128 * NCH;  // floats per staged row
+};
+
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
-                                               float* stage, uint64_t* rowp, int cosine,
-                                               int lane) {
+                                               float* stage, int cosine, int lane) {
   constexpr int R = StageRows<NCH>::R;
   constexpr int NBUF = StageRows<NCH>::NBUF;
   constexpr int LR = Log2<R>::value;
   constexpr int G = R < 8 ? R : 8;  // rows per uniform compute group
+  constexpr int SR = Stage<NCH>::STRIDE;
   const int d4 = dpad >> 2;
   float mine = 0.0f;
   uint64_t q01[NCH], q23[NCH];
+  bool mine_chunk[NCH];  // does this lane own 16 B slice c of a row?
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
     q01[c] = f2pack(qv[c].x, qv[c].y);
     q23[c] = f2pack(qv[c].z, qv[c].w);
+    mine_chunk[c] = c * 32 + lane < d4;
   }
-  // lane j resolves candidate j's row address once
-  if (lane < nc) rowp[lane] = reinterpret_cast<uint64_t>(data + (int64_t)cid[lane] * dpad);
-  __syncwarp();
+  // lane j resolves candidate j's row address (plus nothing else) once
+  const uint64_t rowptr =
+      lane < nc ? reinterpret_cast<uint64_t>(data + (int64_t)cid[lane] * dpad) : 0ull;
   const int rounds = (nc + R - 1) / R;
-  // issue round k: one LDGSTS per row per 16 B chunk, into buffer k % NBUF
   const uint32_t stage_s = smem_u32(stage) + 16u * lane;
-  const uint32_t rowbytes = 4u * (uint32_t)dpad;
   auto issue = [&](int k) {
-    const uint32_t dst0 = stage_s + (uint32_t)((k % NBUF) * R) * rowbytes;
+    const uint32_t dst0 = stage_s + (uint32_t)((k % NBUF) * R * SR * 4);
     const int rows = min(R, nc - k * R);
 #pragma unroll
     for (int rr = 0; rr < R; ++rr) {
-      const bool on = rr < rows;
-      const float4* src = reinterpret_cast<const float4*>(rowp[on ? k * R + rr : 0]) + lane;
+      const uint64_t base = __shfl_sync(FULL, rowptr, (k * R + rr) & 31);
+      const float4* src = reinterpret_cast<const float4*>(base) + lane;
 #pragma unroll
       for (int c = 0; c < NCH; ++c)
-        cp_async16_if(on && (c * 32 + lane < d4), dst0 + rr * rowbytes + 512u * c, src + c * 32);
+        cp_async16_if(rr < rows && mine_chunk[c], dst0 + (uint32_t)(rr * SR * 4 + 512 * c),
+                      src + c * 32);
     }
     cp_async_commit();
   };
@@ -535,18 +545,18 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     const int rows = min(R, nc - b);
     cp_async_wait_pending(min(NBUF - 1, rounds - 1 - k));
     // ---- compute: lane owns its 16 B slices of every staged row
-    const float* buf = stage + (size_t)(k % NBUF) * R * dpad;
+    const float* buf = stage + (size_t)(k % NBUF) * R * SR;
     float part[R];
 #pragma unroll
     for (int g = 0; g < R; g += G) {
       if (g < rows) {
-        const float4* row = reinterpret_cast<const float4*>(buf) + (size_t)g * d4 + lane;
 #pragma unroll
-        for (int r = g; r < g + G; ++r, row += d4) {
+        for (int r = g; r < g + G; ++r) {
+          const float4* row = reinterpret_cast<const float4*>(buf + r * SR) + lane;
           uint64_t acc = 0;
 #pragma unroll
           for (int c = 0; c < NCH; ++c)
-            if (c * 32 + lane < d4) acc = acc4<METRIC>(acc, q01[c], q23[c], row[c * 32]);
+            if (mine_chunk[c]) acc = acc4<METRIC>(acc, q01[c], q23[c], row[c * 32]);
           part[r] = f2sum(acc);
         }
       } else {
@@ -581,7 +591,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
   float* stage = reinterpret_cast<float*>(base);                       // staged rows
-  const size_t stage_bytes = (size_t)StageRows<NCH>::NBUF * R * a.dpad * 4;
+  const size_t stage_bytes = (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
   int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
   uint64_t* rowp = keys32 + 32;                                         // 32 row pointers
@@ -651,8 +661,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
     for (int i = lane; i < tslots; i += 32) table[i] = BLOOM ? 0 : EMPTY;
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, rowp, a.cosine,
-                                                lane);
+    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, a.cosine, lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     if (BLOOM)
       bs.insert(a.entry, lane == 0);
@@ -739,8 +748,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       __syncwarp();
 
       // ---- a5: bulk distance computation (§VI)
-      const float dist = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, rowp,
-                                                    a.cosine, lane);
+      const float dist =
+          bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, a.cosine, lane);
       n_dist += nc;
       n_exp += 1;
 

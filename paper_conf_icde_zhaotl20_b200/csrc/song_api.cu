@@ -192,7 +192,7 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
   const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
-  const int stage_bytes = SONG_STAGE_BUFS * rows * dpad * 4;
+  const int stage_bytes = SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE rows
   s.warp_bytes = stage_bytes + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
