@@ -501,6 +501,33 @@ struct Stage {
   static constexpr int STRIDE = 128 * NCH;  // floats per staged row
 };
 
+// first chunk: no accumulator input (FMUL2 instead of a zeroed FFMA2)
+template <int METRIC>
+__device__ __forceinline__ uint64_t acc4_first(uint64_t q01, uint64_t q23, float4 x) {
+  const uint64_t x01 = f2pack(x.x, x.y), x23 = f2pack(x.z, x.w);
+  uint64_t acc;
+  if (METRIC == MET_L2) {
+    uint64_t d01, d23;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d01) : "l"(q01), "l"(x01));
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d23) : "l"(q23), "l"(x23));
+    asm("mul.rn.f32x2 %0, %1, %1;" : "=l"(acc) : "l"(d01));
+    asm("fma.rn.f32x2 %0, %1, %1, %0;" : "+l"(acc) : "l"(d23));
+  } else {
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(acc) : "l"(q01), "l"(x01));
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(q23), "l"(x23));
+  }
+  return acc;
+}
+
+// zero this lane's slices of every staged row once per launch: slices past
+// dpad are never written by the copies, so they keep contributing 0
+template <int NCH>
+__device__ __forceinline__ void zero_stage(float* stage, int rows, int lane) {
+  float4* s4 = reinterpret_cast<float4*>(stage);
+  for (int i = lane; i < rows * 32 * NCH; i += 32) s4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  __syncwarp();
+}
+
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
@@ -553,10 +580,10 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
 #pragma unroll
         for (int r = g; r < g + G; ++r) {
           const float4* row = reinterpret_cast<const float4*>(buf + r * SR) + lane;
-          uint64_t acc = 0;
+          // (slices past dpad stay zero in the stage and in the query: they add 0)
+          uint64_t acc = acc4_first<METRIC>(q01[0], q23[0], row[0]);
 #pragma unroll
-          for (int c = 0; c < NCH; ++c)
-            if (mine_chunk[c]) acc = acc4<METRIC>(acc, q01[c], q23[c], row[c * 32]);
+          for (int c = 1; c < NCH; ++c) acc = acc4<METRIC>(acc, q01[c], q23[c], row[c * 32]);
           part[r] = f2sum(acc);
         }
       } else {
@@ -604,6 +631,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   HashSet hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};
   const unsigned lt = lanemask_lt();
+  zero_stage<NCH>(stage, StageRows<NCH>::NBUF * R, lane);
 
   while (true) {
     int qi = 0;

@@ -48,7 +48,7 @@ for k, r in enumerate(data):
     agg[line_of[k][0]][0] += float(r[iex] or 0)
     agg[line_of[k][0]][1] += float(r[ist] or 0)
 src = {}
-for (f, n), (e, s) in sorted(agg.items(), key=lambda x: -x[1][0])[:60]:
+for (f, n), (e, s) in sorted(agg.items(), key=lambda x: -x[1][0])[:(100000 if "--all" in sys.argv else 60)]:
     path = None
     for root in ("paper_conf_icde_zhaotl20_b200/csrc",):
         p = os.path.join(root, f) if f else None
