@@ -547,9 +547,11 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     q23[c] = f2pack(qv[c].z, qv[c].w);
     mine_chunk[c] = c * 32 + lane < d4;
   }
-  // lane j resolves candidate j's row address (plus nothing else) once
-  const uint64_t rowptr =
-      lane < nc ? reinterpret_cast<uint64_t>(data + (int64_t)cid[lane] * dpad) : 0ull;
+  // lane j holds candidate j's id; a row's address for this lane is one
+  // IMAD.WIDE: id * rowbytes + (data + 16 B * lane)
+  const uint32_t myid = lane < nc ? (uint32_t)cid[lane] : 0u;
+  const uint32_t rowbytes = 4u * (uint32_t)dpad;
+  const char* lane_base = reinterpret_cast<const char*>(data) + 16 * lane;
   const int rounds = (nc + R - 1) / R;
   const uint32_t stage_s = smem_u32(stage) + 16u * lane;
   auto issue = [&](int k) {
@@ -557,8 +559,8 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     const int rows = min(R, nc - k * R);
 #pragma unroll
     for (int rr = 0; rr < R; ++rr) {
-      const uint64_t base = __shfl_sync(FULL, rowptr, (k * R + rr) & 31);
-      const float4* src = reinterpret_cast<const float4*>(base) + lane;
+      const uint32_t id = __shfl_sync(FULL, myid, (k * R + rr) & 31);
+      const float4* src = reinterpret_cast<const float4*>(lane_base + (uint64_t)id * rowbytes);
 #pragma unroll
       for (int c = 0; c < NCH; ++c)
         cp_async16_if(rr < rows && mine_chunk[c], dst0 + (uint32_t)(rr * SR * 4 + 512 * c),
