@@ -6,7 +6,7 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R8 it follows are listed in its header and in DESIGN.md §3).
+R1-R10 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
@@ -34,8 +34,12 @@ BOUNDED_Q = 1
 SEL = 2
 DEL = 4
 BLOOM = 8
+CUCKOO = 16
 OPTIMIZED = BOUNDED_Q | SEL | DEL          # "hashtable-sel-del" (Fig. 7)
 OPTIMIZED_BLOOM = BOUNDED_Q | SEL | BLOOM  # "bloomfilter" (Fig. 7)
+OPTIMIZED_CUCKOO = BOUNDED_Q | SEL | DEL | CUCKOO  # "cuckoofilter" (Fig. 7)
+HASHTABLE = BOUNDED_Q                      # "hashtable" (Fig. 7): no sel, no del
+HASHTABLE_SEL = BOUNDED_Q | SEL            # "hashtable-sel" (Fig. 7)
 
 _TRACE_FN = ctypes.CFUNCTYPE(
     None, ctypes.c_void_p, ctypes.c_int64,
@@ -71,6 +75,9 @@ def _load():
         lib.oracle_bruteforce.restype = None
         lib.oracle_bruteforce.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                           P, ctypes.c_int64, ctypes.c_int32, P, P, ctypes.c_int32]
+        lib.oracle_cuckoo_probe.restype = ctypes.c_int64
+        lib.oracle_cuckoo_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
+                                            ctypes.c_int64, P]
         lib.oracle_bloom_probe.restype = None
         lib.oracle_bloom_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
                                            ctypes.c_int64, P]
@@ -90,6 +97,23 @@ def _ptr(a):
     return a.ctypes.data_as(ctypes.c_void_p)
 
 
+def default_cuckoo_buckets(L: int) -> int:
+    """DESIGN.md reading R10: 4-slot buckets, >= 4x the live bound 2L + 32."""
+    slots = 1 << int(np.ceil(np.log2(4 * (2 * L + 32))))
+    return slots // 4
+
+
+def cuckoo_probe(buckets: int, ops, probes):
+    """Apply ops (id >= 0 insert, -(id+1) erase) then probe membership."""
+    lib = _load()
+    o = np.ascontiguousarray(ops, np.int64)
+    pr = _i32(probes)
+    out = np.empty(pr.shape[0], np.uint8)
+    drops = lib.oracle_cuckoo_probe(int(buckets), _ptr(o), o.shape[0], _ptr(pr), pr.shape[0],
+                                    _ptr(out))
+    return out.astype(bool), int(drops)
+
+
 def default_bloom_bits(L: int) -> int:
     """DESIGN.md reading A11: m = 2^ceil(log2(10 * 8L)) bits."""
     need = 10 * 8 * L
@@ -100,7 +124,8 @@ def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OP
            bloom_bits: Optional[int] = None, entry: int = 0, max_iters: int = 1 << 40,
            nthreads: int = 1, trace: Optional[Callable] = None):
     """Run the oracle.  Returns (ids [nq,K] int32, dists [nq,K] f32,
-    counters [nq,2] int64 = (n_dist, n_exp), n_capped)."""
+    counters [nq,2] int64 = (n_dist, n_exp), n_capped).  ``bloom_bits`` is the
+    Bloom filter's bit count, or the Cuckoo filter's bucket count."""
     lib = _load()
     data = _f32(data)
     adj = _i32(adj)
@@ -116,7 +141,7 @@ def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OP
     dists = np.empty((nq, K), np.float32)
     counters = np.empty((nq, 2), np.int64)
     if bloom_bits is None:
-        bloom_bits = default_bloom_bits(L)
+        bloom_bits = default_cuckoo_buckets(L) if flags & CUCKOO else default_bloom_bits(L)
     cb = _TRACE_FN()
     if trace is not None:
         def _cb(ctx, it, qp, nqq, tp, nt, vp, nv):

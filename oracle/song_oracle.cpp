@@ -28,6 +28,11 @@
 //   R8 Bloom filter: k = 7 bits per id by double hashing
 //      bit_i = (h1 + i*h2) mod m, h1 = fmix32(id), h2 = fmix32(id ^ 0x5bd1e995) | 1,
 //      fmix32 = MurmurHash3's 32-bit finaliser.  No deletion.
+//   R9 maintenance is a batch: selected candidates are inserted in candidate
+//      order, then q's maximum is evicted while |q| > L (identical sets to the
+//      per-candidate interleaving for exact visited sets; fixes the operation
+//      order for the probabilistic filters).
+//   R10 Cuckoo filter: see struct Cuckoo.
 //
 // Parity status: every function below is pinned by tests/test_oracle_*.py
 // (Fig. 1 / Fig. 4(c) traces, plain == optimized equivalence, brute-force
@@ -54,6 +59,7 @@ enum Flags {
   ORACLE_SEL = 2,        // §IV-D: selected insertion
   ORACLE_DEL = 4,        // §IV-E: visited deletion
   ORACLE_BLOOM = 8,      // §IV-B: visited is a Bloom filter (no deletion)
+  ORACLE_CUCKOO = 16,    // visited is a Cuckoo filter (supports deletion)
 };
 
 struct Key {
@@ -134,22 +140,89 @@ struct Bloom {
   }
 };
 
-// The visited set: an exact hash set, or a Bloom filter.
+// R10: the Cuckoo filter of P:437 [14] ("supports deletion, so it works with
+// visited deletion").  B = 2^b buckets of 4 slots holding 16-bit fingerprints
+// (0 = empty); fp(v) = fmix32(v ^ 0x2545f491) & 0xffff, 0 -> 1;
+// i1 = fmix32(v) mod B, i2 = (i1 ^ fmix32(fp)) mod B (partial-key cuckoo).
+// insert: first empty slot of i1, else of i2, else kick: cur = i2, for
+// n = 0..499 swap with slot n % 4 of cur, cur = alt(cur, fp'), stop at an empty
+// slot; after 500 kicks the homeless fingerprint is dropped (counted).
+// erase: clear the first slot holding fp in i1, else in i2.
+struct Cuckoo {
+  std::vector<uint16_t> slot;  // 4 * B
+  uint32_t mask;
+  int64_t drops = 0;
+  explicit Cuckoo(uint64_t buckets) : slot(4 * buckets, 0), mask((uint32_t)buckets - 1) {}
+  static uint16_t fp(int32_t v) {
+    uint16_t f = (uint16_t)(fmix32((uint32_t)v ^ 0x2545f491u) & 0xffffu);
+    return f ? f : 1;
+  }
+  uint32_t alt(uint32_t i, uint16_t f) const { return (i ^ fmix32((uint32_t)f)) & mask; }
+  bool in_bucket(uint32_t b, uint16_t f) const {
+    for (int j = 0; j < 4; ++j)
+      if (slot[4 * b + j] == f) return true;
+    return false;
+  }
+  bool put(uint32_t b, uint16_t f) {
+    for (int j = 0; j < 4; ++j)
+      if (slot[4 * b + j] == 0) {
+        slot[4 * b + j] = f;
+        return true;
+      }
+    return false;
+  }
+  bool contains(int32_t v) const {
+    const uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask;
+    return in_bucket(i1, f) || in_bucket(alt(i1, f), f);
+  }
+  void insert(int32_t v) {
+    uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask;
+    const uint32_t i2 = alt(i1, f);
+    if (put(i1, f) || put(i2, f)) return;
+    uint32_t cur = i2;
+    for (int n = 0; n < 500; ++n) {
+      std::swap(f, slot[4 * cur + (n & 3)]);
+      cur = alt(cur, f);
+      if (put(cur, f)) return;
+    }
+    ++drops;
+  }
+  void erase(int32_t v) {
+    const uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask;
+    for (uint32_t b : {i1, alt(i1, f)})
+      for (int j = 0; j < 4; ++j)
+        if (slot[4 * b + j] == f) {
+          slot[4 * b + j] = 0;
+          return;
+        }
+  }
+};
+
+// The visited set: an exact hash set, a Bloom filter or a Cuckoo filter.
 struct Visited {
-  bool bloom;
+  int kind;  // 0 exact, 1 Bloom, 2 Cuckoo
   std::unordered_set<int32_t> exact;
   Bloom filter;
-  Visited(bool use_bloom, uint64_t bloom_bits)
-      : bloom(use_bloom), filter(use_bloom ? bloom_bits : 1) {}
-  bool contains(int32_t v) const { return bloom ? filter.contains(v) : exact.count(v) != 0; }
+  Cuckoo cuckoo;
+  Visited(int k, uint64_t bloom_bits, uint64_t cuckoo_buckets)
+      : kind(k), filter(k == 1 ? bloom_bits : 1), cuckoo(k == 2 ? cuckoo_buckets : 1) {}
+  bool contains(int32_t v) const {
+    return kind == 1 ? filter.contains(v) : kind == 2 ? cuckoo.contains(v) : exact.count(v) != 0;
+  }
   void insert(int32_t v) {
-    if (bloom)
+    if (kind == 1)
       filter.insert(v);
+    else if (kind == 2)
+      cuckoo.insert(v);
     else
       exact.insert(v);
   }
   void erase(int32_t v) {
-    if (!bloom) exact.erase(v);  // a Bloom filter cannot delete
+    if (kind == 0) exact.erase(v);
+    if (kind == 2) cuckoo.erase(v);  // a Bloom filter cannot delete
   }
 };
 
@@ -163,8 +236,8 @@ void emit_trace(trace_fn cb, void* ctx, int64_t it, const std::set<Key>& q,
   std::vector<int32_t> qi, ti, vi;
   for (const Key& k : q) qi.push_back(k.id);
   for (const Key& k : topk) ti.push_back(k.id);
-  int64_t nv = -1;  // a Bloom filter cannot be enumerated
-  if (!vis.bloom) {
+  int64_t nv = -1;  // a Bloom / Cuckoo filter cannot be enumerated
+  if (vis.kind == 0) {
     vi.assign(vis.exact.begin(), vis.exact.end());
     std::sort(vi.begin(), vi.end());
     nv = (int64_t)vi.size();
@@ -180,7 +253,7 @@ struct Problem {
   int degree;
   int metric;
   int K, L, flags, entry;
-  uint64_t bloom_bits;
+  uint64_t bloom_bits;  // Bloom: bits; Cuckoo: buckets
   int64_t max_iters;
 };
 
@@ -193,7 +266,8 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
   const bool bounded = P.flags & ORACLE_BOUNDED_Q;
   const bool sel = P.flags & ORACLE_SEL;
   const bool del = P.flags & ORACLE_DEL;
-  Visited visited((P.flags & ORACLE_BLOOM) != 0, P.bloom_bits);
+  Visited visited((P.flags & ORACLE_BLOOM) ? 1 : (P.flags & ORACLE_CUCKOO) ? 2 : 0, P.bloom_bits,
+                  P.bloom_bits);
   std::set<Key> q;     // min-priority queue (begin() = min, prev(end()) = max)
   std::set<Key> topk;  // bounded max-priority queue (R1)
   int64_t n_dist = 0, n_exp = 0;
@@ -246,18 +320,21 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
     for (int32_t v : cand) ck.push_back(Key{distance(p, P.data + (int64_t)v * P.dim, P.dim, P.metric), v});
     n_dist += (int64_t)cand.size();
     n_exp += 1;
-    // 2.6 — maintenance, lines 12-13 with §IV-C/D/E.
+    // 2.6 — maintenance, lines 12-13 with §IV-C/D/E, as a batch (R9: "the data
+    // structure maintenance stage uses the distances to update the priority
+    // queues and the hash table"): insert the selected candidates in
+    // candidate order, then evict q's maximum while |q| > L.
     for (const Key& k : ck) {
       // [sel] P:429: filtered when topk is full and k is worse than all of it (R3).
       if (sel && (int)topk.size() == L && *std::prev(topk.end()) < k) continue;
       visited.insert(k.id);
       q.insert(k);
-      // [bounded] P:421: pop the worst once q grows past L (R4); [del] P:435.
-      if (bounded && (int)q.size() > L) {
-        Key w = *std::prev(q.end());
-        q.erase(std::prev(q.end()));
-        if (del) visited.erase(w.id);
-      }
+    }
+    // [bounded] P:421: pop the worst once q grows past L (R4); [del] P:435.
+    while (bounded && (int)q.size() > L) {
+      Key w = *std::prev(q.end());
+      q.erase(std::prev(q.end()));
+      if (del) visited.erase(w.id);
     }
     emit_trace(cb, ctx, it, q, topk, visited);
   }
@@ -349,6 +426,22 @@ void oracle_bruteforce(const float* data, int64_t n, int32_t dim, int32_t metric
       for (int64_t i = t; i < nq; i += nthreads) one(i);
     });
   for (auto& th : pool) th.join();
+}
+
+// Cuckoo filter probe for tests of R10: applies ops[i] (+id = insert,
+// -(id+1) = erase) in order, then writes 1/0 membership of probe[] to out;
+// returns the number of dropped fingerprints.
+int64_t oracle_cuckoo_probe(int64_t buckets, const int64_t* ops, int64_t nops,
+                            const int32_t* probe, int64_t nprobe, uint8_t* out) {
+  Cuckoo c((uint64_t)buckets);
+  for (int64_t i = 0; i < nops; ++i) {
+    if (ops[i] >= 0)
+      c.insert((int32_t)ops[i]);
+    else
+      c.erase((int32_t)(-ops[i] - 1));
+  }
+  for (int64_t i = 0; i < nprobe; ++i) out[i] = c.contains(probe[i]) ? 1 : 0;
+  return c.drops;
 }
 
 // Bloom filter probe for tests of §IV-B: inserts ins[0..nins), then
