@@ -52,13 +52,22 @@ typedef enum {
                              dim > 1024, queue_len > SONG_MAX_QUEUE_LEN,
                              shared-memory budget exceeded) */
   SONG_EITERCAP = -5      /* a query reached params.max_iters expansions */
+  /* (SONG_EUNSUPPORTED is also the sticky status of a query whose global
+     visited table filled up; raise params.table_log2) */
 } song_status;
 
 typedef enum {
-  SONG_VISITED_HASH = 0,  /* open addressing, selected insertion + visited deletion
-                             ("hashtable-sel-del", Fig. 7) */
-  SONG_VISITED_BLOOM = 1  /* Bloom filter, selected insertion, no deletion
-                             ("bloomfilter") */
+  SONG_VISITED_HASH = 0,            /* shared-memory open addressing, selected insertion +
+                                       visited deletion ("hashtable-sel-del", Fig. 7)
+                                       — the default and the fast path */
+  SONG_VISITED_BLOOM = 1,           /* shared-memory Bloom filter, selected insertion, no
+                                       deletion ("bloomfilter") */
+  SONG_VISITED_HASH_GLOBAL = 2,     /* exact hash in global memory, no selected insertion,
+                                       no deletion ("hashtable", Fig. 7) */
+  SONG_VISITED_HASH_GLOBAL_SEL = 3, /* as 2 with selected insertion ("hashtable-sel") */
+  SONG_VISITED_CUCKOO = 4           /* shared-memory Cuckoo filter, selected insertion +
+                                       visited deletion ("cuckoofilter"; DESIGN.md
+                                       reading R10) */
 } song_visited_kind;
 
 #define SONG_MAX_DEGREE 32
@@ -78,7 +87,11 @@ typedef struct song_search_params {
   int32_t blocks_per_sm;   /* launch shape: 0 = as many as fit */
   int32_t id_offset;       /* added to every returned id (dataset sharding, P:471:
                               shard-local ids become global ids); default 0 */
-  int32_t reserved;        /* must be 0 */
+  int32_t table_log2;      /* capacity of the visited table: HASH_GLOBAL(_SEL): log2
+                              slots per warp (default max(14, ceil(log2(64 L)))); a
+                              query that fills half of it stops with SONG_EUNSUPPORTED
+                              status; CUCKOO: log2 buckets of 4 (default: 4 slots per
+                              live key bound 2L+32); ignored otherwise; 0 = default */
 } song_search_params;
 
 typedef struct song_index_info {

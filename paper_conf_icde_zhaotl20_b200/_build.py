@@ -1,4 +1,10 @@
-"""Compile libsong.so (the C-ABI library of include/song.h) for sm_100a, in-tree."""
+"""Compile libsong.so (the C-ABI library of include/song.h) for sm_100a, in-tree.
+
+The kernel variants are split over one translation unit per row width
+(csrc/launch_nch{1,2,4,8}.cu) and compiled in parallel, then linked with the
+C-ABI (csrc/song_api.cu) into one shared library.
+"""
+import concurrent.futures
 import os
 import subprocess
 import sys
@@ -6,35 +12,52 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
+BUILD = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libsong.so")
-SOURCES = [os.path.join(CSRC, "song_api.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in os.listdir(CSRC)] + [
-    os.path.join(ROOT, "include", "song.h")]
+SOURCES = ["song_api.cu", "launch_nch1.cu", "launch_nch2.cu", "launch_nch4.cu", "launch_nch8.cu"]
+DEPS = [os.path.join(CSRC, f) for f in os.listdir(CSRC)] + [os.path.join(ROOT, "include", "song.h")]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17",
-    "-Xcompiler", "-fPIC", "-shared",
+    "-Xcompiler", "-fPIC",
     "-Xptxas", "-v",
 ]
+
+
+def _compile(src):
+    obj = os.path.join(BUILD, src.replace(".cu", ".o"))
+    cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-c",
+           "-o", obj, os.path.join(CSRC, src)]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    return src, obj, res
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
     newest = max(os.path.getmtime(p) for p in DEPS)
     if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest:
         return LIB
-    cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-I", CSRC,
-           "-o", LIB, *SOURCES]
-    res = subprocess.run(cmd, capture_output=True, text=True)
+    os.makedirs(BUILD, exist_ok=True)
+    with concurrent.futures.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
+        results = list(ex.map(_compile, SOURCES))
+    report = []
+    for src, obj, res in results:
+        if res.returncode != 0:
+            sys.stderr.write(res.stdout + res.stderr)
+            raise RuntimeError(f"nvcc failed compiling {src}")
+        report.append(res.stderr)
+    link = ["nvcc", "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", LIB,
+            *[obj for _, obj, _ in results]]
+    res = subprocess.run(link, capture_output=True, text=True)
     if res.returncode != 0:
         sys.stderr.write(res.stdout + res.stderr)
-        raise RuntimeError("nvcc failed building libsong.so")
+        raise RuntimeError("nvcc failed linking libsong.so")
     with open(os.path.join(PKG, "ptxas_report.txt"), "w") as f:
-        f.write(res.stderr)
+        f.write("\n".join(report))
     if verbose:
-        sys.stderr.write(res.stderr)
+        sys.stderr.write("\n".join(report))
     return LIB
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose=True))
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

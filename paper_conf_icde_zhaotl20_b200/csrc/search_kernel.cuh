@@ -41,7 +41,9 @@ constexpr int TOMB = -2;   // hash slot whose key was deleted (§IV-E)
 constexpr uint64_t KEY_MAX = ~0ull;
 constexpr int STAGE_BYTES = 16384;  // per-warp row stage (32 rows of d = 128)
 
-enum : int { STATUS_BAD_INPUT = 1, STATUS_ITER_CAP = 2 };
+enum : int { STATUS_BAD_INPUT = 1, STATUS_ITER_CAP = 2, STATUS_TABLE_FULL = 4 };
+// visited-set kinds (template parameter VK of the kernel)
+enum : int { VK_HASH = 0, VK_BLOOM = 1, VK_GHASH = 2, VK_CUCKOO = 3 };
 enum : int { MET_L2 = 0, MET_DOT = 1 };
 
 struct SearchArgs {
@@ -62,6 +64,9 @@ struct SearchArgs {
   int cosine;      // MET_DOT: 1 -> 1 - dot, 0 -> -dot
   int dedup;       // 1 if some adjacency row repeats an id
   int rebuild_at;  // hash: rebuild when live + tombstones would exceed this
+  int sel;         // selected insertion on (VK_GHASH: hashtable-sel vs hashtable)
+  uint64_t* gtab;  // VK_GHASH: [grid warps][2^table_log2] u64
+  uint32_t gen0;   // VK_GHASH: generation base of this launch
   int warp_smem_bytes;
 };
 
@@ -219,6 +224,124 @@ struct BloomSet {
       }
     }
     __syncwarp();
+  }
+};
+
+// Exact visited set in GLOBAL memory for the variants without visited
+// deletion ("hashtable" / "hashtable-sel" of Fig. 7; the paper keeps
+// the unbounded table in global memory).  One table of 2^log2 u64 slots
+// per resident warp; a slot holds (generation << 32 | id) and counts as empty
+// unless its generation is the current query's, so tables are never cleared.
+struct GHash {
+  uint64_t* slot;
+  int log2;
+  uint32_t gen;
+  __device__ __forceinline__ unsigned home(int v) const {
+    return ((uint32_t)v * 0x9E3779B1u) >> (32 - log2);
+  }
+  __device__ __forceinline__ bool contains(int v, bool act) const {
+    const unsigned mask = (1u << log2) - 1;
+    const uint64_t want = ((uint64_t)gen << 32) | (uint32_t)v;
+    unsigned h = home(v);
+    bool found = false;
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const uint64_t s = slot[h];
+        found = (s == want);
+        act = !found && (uint32_t)(s >> 32) == gen;
+        h = (h + 1) & mask;
+      }
+    }
+    return found;
+  }
+  __device__ __forceinline__ void insert(int v, bool act) {
+    const unsigned mask = (1u << log2) - 1;
+    const uint64_t want = ((uint64_t)gen << 32) | (uint32_t)v;
+    unsigned h = home(v);
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const uint64_t s = slot[h];
+        if ((uint32_t)(s >> 32) != gen) {
+          const unsigned long long old =
+              atomicCAS(reinterpret_cast<unsigned long long*>(slot + h), (unsigned long long)s,
+                        (unsigned long long)want);
+          if (old == s) act = false;  // else: lost the race, re-read the slot
+        } else {
+          h = (h + 1) & mask;
+        }
+      }
+    }
+  }
+};
+
+// Cuckoo filter (reading R10; the oracle's struct Cuckoo): 2^log2
+// buckets of 4 x 16-bit fingerprints in shared memory.  Lookups run on all
+// lanes in parallel; inserts and erases are single-lane and issued in the
+// oracle's order (kicks make the state order-dependent).
+struct CuckooSet {
+  uint16_t* slot;
+  int log2;
+  __device__ __forceinline__ uint32_t mask() const { return (1u << log2) - 1; }
+  __device__ __forceinline__ static uint16_t fp(int v) {
+    const uint16_t f = (uint16_t)(fmix32((uint32_t)v ^ 0x2545f491u) & 0xffffu);
+    return f ? f : (uint16_t)1;
+  }
+  __device__ __forceinline__ uint32_t alt(uint32_t i, uint16_t f) const {
+    return (i ^ fmix32((uint32_t)f)) & mask();
+  }
+  __device__ __forceinline__ bool in_bucket(uint32_t b, uint16_t f) const {
+    const uint2 w = reinterpret_cast<const uint2*>(slot)[b];  // 4 fingerprints
+    const uint32_t ff = (uint32_t)f;
+    return ((w.x & 0xffffu) == ff) | ((w.x >> 16) == ff) | ((w.y & 0xffffu) == ff) |
+           ((w.y >> 16) == ff);
+  }
+  __device__ __forceinline__ bool contains(int v, bool act) const {
+    if (!act) return false;
+    const uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask();
+    return in_bucket(i1, f) || in_bucket(alt(i1, f), f);
+  }
+  __device__ __forceinline__ bool put(uint32_t b, uint16_t f) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (slot[4 * b + j] == 0) {
+        slot[4 * b + j] = f;
+        return true;
+      }
+    return false;
+  }
+  // single lane; returns false when a fingerprint was dropped after 500 kicks
+  __device__ __forceinline__ bool insert1(int v) {
+    uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask();
+    const uint32_t i2 = alt(i1, f);
+    if (put(i1, f) || put(i2, f)) return true;
+    uint32_t cur = i2;
+    for (int n = 0; n < 500; ++n) {
+      const uint16_t victim = slot[4 * cur + (n & 3)];
+      slot[4 * cur + (n & 3)] = f;
+      f = victim;
+      cur = alt(cur, f);
+      if (put(cur, f)) return true;
+    }
+    return false;
+  }
+  __device__ __forceinline__ void erase1(int v) {
+    const uint16_t f = fp(v);
+    const uint32_t i1 = fmix32((uint32_t)v) & mask();
+    const uint32_t b2 = alt(i1, f);
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (slot[4 * i1 + j] == f) {
+        slot[4 * i1 + j] = 0;
+        return;
+      }
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (slot[4 * b2 + j] == f) {
+        slot[4 * b2 + j] = 0;
+        return;
+      }
   }
 };
 
@@ -611,10 +734,11 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
 #define SONG_LB_BLOCKS 6
 #endif
 // QR > 0: q / topk in registers (queue_len <= 32*QR); QR == 0: shared memory.
-template <int NCH, int METRIC, bool BLOOM, int QR>
+template <int NCH, int METRIC, int VK, int QR>
 __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH>::R;
+  constexpr bool DEL = (VK == VK_HASH || VK == VK_CUCKOO);  // visited deletion (§IV-E)
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int L = a.L;
@@ -623,18 +747,60 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   const size_t stage_bytes = (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
   int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
-  uint64_t* rowp = keys32 + 32;                                         // 32 row pointers
-  uint64_t* qa = rowp + 32;                                             // QR == 0 only
+  uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
+  uint64_t* qa = ev + 32;                                               // QR == 0 only
   uint64_t* qb = qa + (QR == 0 ? L : 0);
   uint64_t* tk = qb + (QR == 0 ? L : 0);
   int* table = reinterpret_cast<int*>(                                  // 16 B aligned
       (reinterpret_cast<uintptr_t>(tk + (QR == 0 ? L : 0)) + 15) & ~uintptr_t(15));
-  const int tslots = BLOOM ? ((1 << a.table_log2) >> 5) : (1 << a.table_log2);
+  // 32-bit words of the shared-memory visited table
+  const int twords = VK == VK_HASH    ? (1 << a.table_log2)
+                     : VK == VK_BLOOM ? ((1 << a.table_log2) >> 5)
+                     : VK == VK_CUCKOO ? (2 << a.table_log2)  // 4 x u16 per bucket
+                                       : 0;
   HashSet hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};
+  CuckooSet cs{reinterpret_cast<uint16_t*>(table), a.table_log2};
+  GHash gh{a.gtab + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2),
+           a.table_log2, a.gen0};
   const unsigned lt = lanemask_lt();
   zero_stage<NCH>(stage, StageRows<NCH>::NBUF * R, lane);
 
+  // ---- visited-set operations (§IV-B/D/E) for the four kinds
+  auto v_contains = [&](int v, bool act) -> bool {
+    if constexpr (VK == VK_HASH) return hs.contains(v, act);
+    if constexpr (VK == VK_BLOOM) return bs.contains(v, act);
+    if constexpr (VK == VK_GHASH) return gh.contains(v, act);
+    if constexpr (VK == VK_CUCKOO) return cs.contains(v, act);
+    return false;
+  };
+  // single-lane insert / erase (entry vertex, topk eviction)
+  auto v_insert_lane0 = [&](int v) {
+    if constexpr (VK == VK_HASH) hs.insert(v, lane == 0);
+    if constexpr (VK == VK_BLOOM) bs.insert(v, lane == 0);
+    if constexpr (VK == VK_GHASH) gh.insert(v, lane == 0);
+    if constexpr (VK == VK_CUCKOO) {
+      if (lane == 0) cs.insert1(v);
+      __syncwarp();
+    }
+  };
+  auto v_erase_lane0 = [&](uint64_t k) {
+    if constexpr (VK == VK_HASH) hs.erase(key_id(k), k != KEY_MAX && lane == 0);
+    if constexpr (VK == VK_CUCKOO) {
+      if (lane == 0 && k != KEY_MAX) cs.erase1(key_id(k));
+      __syncwarp();
+    }
+  };
+  // Cuckoo: erase the evicted keys ev[0..ne) one at a time in decreasing key
+  // order (reading R9's eviction order)
+  auto cuckoo_erase_sorted_desc = [&](int ne) {
+    for (int i = ne - 1; i >= 0; --i) {
+      if (lane == 0) cs.erase1(key_id(ev[i]));
+      __syncwarp();
+    }
+  };
+
+  uint32_t gen = a.gen0;
   while (true) {
     int qi = 0;
     if (lane == 0) qi = (int)atomicAdd(a.ticket, 1u);
@@ -688,16 +854,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
     }
 
     // ---- a2: init — visited = {e}, q = {(d_e, e)}, topk = {} (Alg. 1 line 1)
-    for (int i = lane; i < tslots; i += 32) table[i] = BLOOM ? 0 : EMPTY;
+    for (int i = lane; i < twords; i += 32) table[i] = VK == VK_HASH ? EMPTY : 0;
+    if (VK == VK_GHASH) gh.gen = ++gen;  // a fresh generation empties the table
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
     const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, a.cosine, lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
-    if (BLOOM)
-      bs.insert(a.entry, lane == 0);
-    else
-      hs.insert(a.entry, lane == 0);
-    int used = 1;
+    v_insert_lane0(a.entry);
+    int used = 1;  // VK_HASH: live + tombstones; VK_GHASH: live
     RegArr<QR == 0 ? 1 : QR> q, tk_r;
     q.clear();
     tk_r.clear();
@@ -708,7 +872,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
     }
     int qsize = 1, tsize = 0;
     int n_dist = 1, n_exp = 0, iters = 0;
-    bool capped = false;
+    bool capped = false, full = false;
     // adjacency row of the next head, prefetched (lane j holds slot j)
     int adjv = (lane < a.degree) ? __ldg(a.adj + (int64_t)a.entry * a.degree + lane) : -1;
     __syncwarp();
@@ -730,10 +894,23 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       }
       if (tmax < now) break;  // topk full and its max beats now (lines 4-5)
       uint64_t evicted = KEY_MAX;
+      // Cuckoo false negatives can re-admit a vertex that is already in topk:
+      // topk then stays as it is (the paper's "additional checks to avoid
+      // inserting one vertex multiple times"; the oracle's set semantics)
+      bool in_topk = false;
+      if constexpr (VK == VK_CUCKOO) {
+        if (QR > 0) {
+#pragma unroll
+          for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) in_topk |= __any_sync(FULL, tk_r.v[r] == now);
+        } else {
+          for (int b0 = 0; b0 < tsize; b0 += 32)
+            in_topk |= __any_sync(FULL, b0 + lane < tsize && tk[b0 + lane] == now);
+        }
+      }
       if (QR > 0) {
-        evicted = tk_r.insert_one(now, L, lane);
+        if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
         q.pop_front(lane);
-      } else {
+      } else if (!in_topk) {
         evicted = (tsize == L) ? tk[L - 1] : KEY_MAX;
         int pos = 0;
         for (int b0 = 0; b0 < tsize; b0 += 32) {
@@ -756,8 +933,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
           if (w) tk[i] = val;
         }
       }
-      tsize = min(tsize + 1, L);
-      if (!BLOOM) hs.erase(key_id(evicted), evicted != KEY_MAX && lane == 0);  // §IV-E
+      if (!in_topk) tsize = min(tsize + 1, L);
+      if (DEL) v_erase_lane0(evicted);  // §IV-E: topk's evicted vertex
       __syncwarp();
       const int na = qsize - 1;  // q after the pop
       const uint64_t* A = qa + 1;
@@ -770,7 +947,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
         keep = keep && ((grp & lt) == 0);
       }
       // (called by every lane: the probe loops are warp-collective)
-      const bool seen = BLOOM ? bs.contains(v, keep) : hs.contains(v, keep);
+      const bool seen = v_contains(v, keep);
       keep = keep && !seen;
       const unsigned km = __ballot_sync(FULL, keep);
       const int nc = __popc(km);
@@ -786,8 +963,11 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cid[lane] : -1;
       uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
-      const uint64_t thr = (tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
-      const bool sel = (lane < nc) && key < thr;  // selected insertion
+      const uint64_t thr =
+          (a.sel && tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
+      // selected insertion: filtered only when worse than ALL of topk
+      // (a key equal to topk's max can only arise from a filter false negative)
+      const bool sel = (lane < nc) && key <= thr;
       const unsigned smask = __ballot_sync(FULL, sel);
       const int ns = __popc(smask);
       if (!sel) key = KEY_MAX;
@@ -795,89 +975,153 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       {
         uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na > 0 ? A[0] : KEY_MAX);
         uint64_t nxt = umin64(qhead, warp_min_key(key));
-#ifdef SONG_DEBUG
-        if (qi == 0 && lane < 32)
-          printf("it %d lane %d now %llx nc %d cid %d dist %f key %llx qhead %llx nxt %llx q0 %llx\n", iters, lane,
-                 (unsigned long long)now, nc, myid, dist, (unsigned long long)key, (unsigned long long)qhead,
-                 (unsigned long long)nxt, (unsigned long long)q.v[0]);
-#endif
         if (nxt != KEY_MAX && lane < a.degree)
           adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
         else
           adjv = -1;
       }
-      // visited insert of the selected candidates (hash: rebuild first when
-      // tombstones accumulated — visited = ids(q) ∪ ids(topk))
+      // visited insert of the selected candidates, in candidate order (R9)
       auto visit_selected = [&]() {
-        if (BLOOM) {
-          bs.insert(myid, sel);
-          return;
+        if constexpr (VK == VK_BLOOM) bs.insert(myid, sel);
+        if constexpr (VK == VK_GHASH) {
+          gh.insert(myid, sel);
+          used += ns;
         }
-        if (used + ns > a.rebuild_at) {
-          for (int i = lane; i < tslots; i += 32) table[i] = EMPTY;
-          __syncwarp();
-          if (QR > 0) {
-#pragma unroll
-            for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
-              hs.insert(key_id(q.v[r]), q.v[r] != KEY_MAX);
-              hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
-            }
-          } else {
-            for (int i0 = 0; i0 < na; i0 += 32)
-              hs.insert(i0 + lane < na ? key_id(A[i0 + lane]) : 0, i0 + lane < na);
-            for (int i0 = 0; i0 < tsize; i0 += 32)
-              hs.insert(i0 + lane < tsize ? key_id(tk[i0 + lane]) : 0, i0 + lane < tsize);
+        if constexpr (VK == VK_CUCKOO) {
+          bool dropped = false;
+          for (unsigned m = smask; m; m &= m - 1) {
+            const int j = __ffs(m) - 1;
+            if (lane == j) dropped |= !cs.insert1(myid);
+            __syncwarp();
           }
-          used = na + tsize;
-          __syncwarp();
+          (void)dropped;  // a dropped fingerprint is a false negative (oracle: drops)
         }
-        const bool took = hs.insert(myid, sel);
-        used += __popc(__ballot_sync(FULL, took));
+        if constexpr (VK == VK_HASH) {
+          if (used + ns > a.rebuild_at) {
+            // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
+            for (int i = lane; i < twords; i += 32) table[i] = EMPTY;
+            __syncwarp();
+            if (QR > 0) {
+#pragma unroll
+              for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+                hs.insert(key_id(q.v[r]), q.v[r] != KEY_MAX);
+                hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
+              }
+            } else {
+              for (int i0 = 0; i0 < na; i0 += 32)
+                hs.insert(i0 + lane < na ? key_id(A[i0 + lane]) : 0, i0 + lane < na);
+              for (int i0 = 0; i0 < tsize; i0 += 32)
+                hs.insert(i0 + lane < tsize ? key_id(tk[i0 + lane]) : 0, i0 + lane < tsize);
+            }
+            used = na + tsize;
+            __syncwarp();
+          }
+          const bool took = hs.insert(myid, sel);
+          used += __popc(__ballot_sync(FULL, took));
+        }
       };
+      int qsize_new = min(na + ns, L);
       if (QR > 0) {
         if (ns > 0) {  // (ns == 0: q only lost its head, nothing to insert/evict)
           visit_selected();
-          // compact the selected keys to lanes [0, ns), sort only those
-          if (sel) keys32[__popc(smask & lt)] = key;
+          // Cuckoo false negatives: a selected key may already be in q
+          unsigned qmask = smask;
+          if constexpr (VK == VK_CUCKOO) {
+            for (unsigned m = smask; m; m &= m - 1) {
+              const int j = __ffs(m) - 1;
+              const uint64_t kj = __shfl_sync(FULL, key, j);
+              bool dup = false;
+#pragma unroll
+              for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) dup |= __any_sync(FULL, q.v[r] == kj);
+              if (dup) qmask &= ~(1u << j);
+            }
+          }
+          const int nq_new = __popc(qmask);
+          qsize_new = min(na + nq_new, L);
+          // compact the selected keys to lanes [0, nq_new), sort only those
+          if ((qmask >> lane) & 1u) keys32[__popc(qmask & lt)] = key;
           __syncwarp();
-          uint64_t k2 = lane < ns ? keys32[lane] : KEY_MAX;
-          k2 = sort_prefix(k2, ns, lane);
+          uint64_t k2 = lane < nq_new ? keys32[lane] : KEY_MAX;
+          k2 = sort_prefix(k2, nq_new, lane);
           const uint64_t sdesc = __shfl_sync(FULL, k2, 31 - lane);  // descending
           // merge into q; evict beyond L (§IV-C) and delete from visited (§IV-E)
           uint64_t out;
           merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
+          int ne = 0;  // number of evicted keys (VK_CUCKOO collects them in ev[])
 #pragma unroll
           for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
-            const bool beyond = r * 32 + lane >= L;
-            if (!BLOOM) hs.erase(key_id(q.v[r]), beyond && q.v[r] != KEY_MAX);
-            q.v[r] = beyond ? KEY_MAX : q.v[r];
+            const bool beyond = r * 32 + lane >= L && q.v[r] != KEY_MAX;
+            if constexpr (VK == VK_HASH) hs.erase(key_id(q.v[r]), beyond);
+            if constexpr (VK == VK_CUCKOO) {
+              const unsigned bm = __ballot_sync(FULL, beyond);
+              if (beyond) ev[ne + __popc(bm & lt)] = q.v[r];
+              ne += __popc(bm);
+            }
+            q.v[r] = r * 32 + lane >= L ? KEY_MAX : q.v[r];
           }
-          if (!BLOOM) hs.erase(key_id(out), out != KEY_MAX);
+          if constexpr (VK == VK_HASH) hs.erase(key_id(out), out != KEY_MAX);
+          if constexpr (VK == VK_CUCKOO) {
+            const bool o = out != KEY_MAX;
+            const unsigned bm = __ballot_sync(FULL, o);
+            if (o) ev[ne + __popc(bm & lt)] = out;
+            ne += __popc(bm);
+            __syncwarp();
+            // sort the evicted keys ascending, erase from the largest down
+            uint64_t e2 = lane < ne ? ev[lane] : KEY_MAX;
+            e2 = sort_prefix(e2, ne, lane);
+            __syncwarp();
+            ev[lane] = e2;
+            __syncwarp();
+            cuckoo_erase_sorted_desc(ne);
+          }
         }
       } else {
         visit_selected();
         __syncwarp();
         key = bitonic_sort32<false>(key, lane);
+        int nsq = ns;  // selected keys that enter q
+        if constexpr (VK == VK_CUCKOO) {
+          // drop keys already in q (Cuckoo false negatives), re-compact
+          const int j = count_below(A, na, key);
+          const bool dup = lane < ns && j < na && A[j] == key;
+          const unsigned keepm = __ballot_sync(FULL, lane < ns && !dup);
+          nsq = __popc(keepm);
+          __syncwarp();
+          if ((keepm >> lane) & 1u) keys32[__popc(keepm & lt)] = key;
+          __syncwarp();
+          key = lane < nsq ? keys32[lane] : KEY_MAX;
+          __syncwarp();
+        }
         keys32[lane] = key;
         __syncwarp();
+        // merged position p >= L is evicted: ev[p - L] (< 32 of them) in key order
         for (int i0 = 0; i0 < na; i0 += 32) {
           const int i = i0 + lane;
           const uint64_t x = i < na ? A[i] : KEY_MAX;
-          const int p = i + count_below(keys32, ns, x);
+          const int p = i + count_below(keys32, nsq, x);
           if (i < na && p < L) qb[p] = x;
-          if (!BLOOM) hs.erase(key_id(x), i < na && p >= L);
+          if (i < na && p >= L) ev[p - L] = x;
+          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na && p >= L);
         }
         {
           const int p = lane + count_below(A, na, key);
-          if (lane < ns && p < L) qb[p] = key;
-          if (!BLOOM) hs.erase(key_id(key), lane < ns && p >= L);
+          if (lane < nsq && p < L) qb[p] = key;
+          if (lane < nsq && p >= L) ev[p - L] = key;
+          if constexpr (VK == VK_HASH) hs.erase(key_id(key), lane < nsq && p >= L);
         }
+        __syncwarp();
+        if constexpr (VK == VK_CUCKOO) cuckoo_erase_sorted_desc(max(0, na + nsq - L));
+        qsize_new = min(na + nsq, L);
         uint64_t* t = qa;
         qa = qb;
         qb = t;
       }
-      qsize = min(na + ns, L);
+      qsize = qsize_new;
       __syncwarp();
+      if (VK == VK_GHASH && used > (1 << (a.table_log2 - 1))) {  // keep load <= 1/2
+        full = true;
+        break;
+      }
     }
 
     // ---- a7: output the first K of topk (Alg. 1 line 17)
@@ -902,7 +1146,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
           dists_o[i] = __int_as_float(0x7f800000);
         }
       }
-      qa = rowp + 32;
+      qa = ev + 32;
       qb = qa + L;
     }
     if (a.counters_out && lane == 0) {
@@ -910,6 +1154,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
       a.counters_out[2 * (int64_t)qi + 1] = n_exp;
     }
     if (capped && lane == 0) atomicOr(a.status, STATUS_ITER_CAP);
+    if (full && lane == 0) atomicOr(a.status, STATUS_TABLE_FULL);
     __syncwarp();
   }
 }

@@ -16,27 +16,9 @@
 #include "search_kernel.cuh"
 #include "song.h"
 
-struct song_index {
-  int device = 0;
-  int num_sms = 0;
-  int64_t n = 0;
-  int dim = 0, dpad = 0, degree = 0, metric = 0;
-  float* d_data = nullptr;
-  int32_t* d_adj = nullptr;
-  unsigned* d_ticket = nullptr;
-  int* d_status = nullptr;
-  int dedup = 1;                       // some adjacency row repeats an id
-  cudaStream_t stream = nullptr;       // owned; used by song_search
-  cudaStream_t last_stream = nullptr;  // stream of the last search
-  // scratch for the host-buffer entry point
-  float* d_q = nullptr;
-  int32_t* d_ids = nullptr;
-  float* d_dists = nullptr;
-  size_t cap_q = 0, cap_out = 0;
-};
+#include "song_internal.h"
 
-namespace {
-
+namespace song {
 thread_local std::string g_err;
 
 int fail(int code, const char* fmt, ...) {
@@ -48,14 +30,21 @@ int fail(int code, const char* fmt, ...) {
   g_err = buf;
   return code;
 }
+}  // namespace song
 
-#define CUDA_TRY(expr)                                                             \
-  do {                                                                             \
-    cudaError_t e_ = (expr);                                                       \
-    if (e_ != cudaSuccess)                                                         \
-      return fail(e_ == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA,      \
-                  "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
-  } while (0)
+namespace song {
+// launch_m<NCH> lives in launch_nch<NCH>.cu (one translation unit per NCH,
+// compiled in parallel)
+template <int NCH>
+int launch_m(song_index* ix, const SearchArgs& a, int metric, int vk, int qr, int warps, int bps,
+             int sms, cudaStream_t st);
+}  // namespace song
+
+namespace {
+using song::fail;
+using song::launch_m;
+using song::g_err;
+
 
 int next_pow2_log2(int64_t x) {
   int l = 0;
@@ -138,6 +127,7 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_q);
   cudaFree(ix->d_ids);
   cudaFree(ix->d_dists);
+  cudaFree(ix->d_gtab);
   if (ix->stream) cudaStreamDestroy(ix->stream);
   delete ix;
 }
@@ -170,14 +160,21 @@ struct Shape {
   int nch;
 };
 
-Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
+Shape search_shape(int L, int vk, const song_search_params* p, int dpad) {
   Shape s;
-  int tbytes;
+  int tbytes = 0;
   s.rebuild_at = 0;
-  if (bloom) {
-    s.table_log2 = bloom_log2_bits > 0 ? bloom_log2_bits : next_pow2_log2(80ll * L);
+  if (vk == song::VK_BLOOM) {
+    s.table_log2 = p->bloom_log2_bits > 0 ? p->bloom_log2_bits : next_pow2_log2(80ll * L);
     if (s.table_log2 < 5) s.table_log2 = 5;
     tbytes = (1 << s.table_log2) / 8;
+  } else if (vk == song::VK_GHASH) {
+    s.table_log2 = p->table_log2 > 0 ? p->table_log2 : std::max(14, next_pow2_log2(64ll * L));
+    tbytes = 0;  // global memory
+  } else if (vk == song::VK_CUCKOO) {
+    // reading R10 default: 4 slots per key of the live bound 2L + 32
+    s.table_log2 = p->table_log2 > 0 ? p->table_log2 : next_pow2_log2(4ll * (2 * L + 32)) - 2;
+    tbytes = (4 << s.table_log2) * 2;
   } else {
     // live keys <= |q| + |topk| + 32 new ones <= 2L + 32.  Register-queue
     // sizes get >= 8x that many slots and rebuild at 1/4 occupancy (about one
@@ -199,59 +196,22 @@ Shape search_shape(int L, bool bloom, int bloom_log2_bits, int dpad) {
   return s;
 }
 
-template <int NCH, int METRIC, bool BLOOM, int QR>
-int launch_t(const song::SearchArgs& a, int warps, int blocks_per_sm, int num_sms,
-             cudaStream_t st) {
-  auto kern = song::song_search_kernel<NCH, METRIC, BLOOM, QR>;
-  const size_t smem = (size_t)a.warp_smem_bytes * warps;
-  CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int fit = 0;
-  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&fit, kern, warps * 32, smem));
-  if (fit < 1) return fail(SONG_EUNSUPPORTED, "search kernel does not fit an SM (%zu B smem)", smem);
-  int bps = blocks_per_sm > 0 ? std::min(blocks_per_sm, fit) : fit;
-  int64_t want = (a.nq + warps - 1) / warps;
-  int64_t grid = std::min<int64_t>((int64_t)bps * num_sms, want);
-  CUDA_TRY(cudaMemsetAsync(a.ticket, 0, sizeof(unsigned), st));
-  kern<<<(unsigned)grid, warps * 32, smem, st>>>(a);
-  CUDA_TRY(cudaGetLastError());
-  return SONG_OK;
-}
-
-template <int NCH, int METRIC, bool BLOOM>
-int launch_q(const song::SearchArgs& a, int qr, int warps, int bps, int sms,
-             cudaStream_t st) {
-  switch (qr) {
-    case 1: return launch_t<NCH, METRIC, BLOOM, 1>(a, warps, bps, sms, st);
-    case 2: return launch_t<NCH, METRIC, BLOOM, 2>(a, warps, bps, sms, st);
-    case 4: return launch_t<NCH, METRIC, BLOOM, 4>(a, warps, bps, sms, st);
-    default: return launch_t<NCH, METRIC, BLOOM, 0>(a, warps, bps, sms, st);
-  }
-}
-
-template <int NCH>
-int launch_m(const song::SearchArgs& a, int metric, bool bloom, int qr,
-             int warps, int bps, int sms, cudaStream_t st) {
-  if (metric == SONG_L2)
-    return bloom ? launch_q<NCH, song::MET_L2, true>(a, qr, warps, bps, sms, st)
-                 : launch_q<NCH, song::MET_L2, false>(a, qr, warps, bps, sms, st);
-  return bloom ? launch_q<NCH, song::MET_DOT, true>(a, qr, warps, bps, sms, st)
-               : launch_q<NCH, song::MET_DOT, false>(a, qr, warps, bps, sms, st);
-}
 
 int check_params(const song_index* ix, const song_search_params* p) {
   if (p->K < 1) return fail(SONG_EINVAL, "K must be >= 1");
   if (p->queue_len < p->K) return fail(SONG_EINVAL, "queue_len %d < K %d", p->queue_len, p->K);
   if (p->queue_len > SONG_MAX_QUEUE_LEN)
     return fail(SONG_EUNSUPPORTED, "queue_len %d > %d", p->queue_len, SONG_MAX_QUEUE_LEN);
-  if (p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM)
+  if (p->visited < SONG_VISITED_HASH || p->visited > SONG_VISITED_CUCKOO)
     return fail(SONG_EINVAL, "unknown visited kind %d", p->visited);
+  if (p->table_log2 < 0 || p->table_log2 > 24)
+    return fail(SONG_EUNSUPPORTED, "table_log2 %d outside [0, 24]", p->table_log2);
   if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
   if (p->bloom_log2_bits < 0 || p->bloom_log2_bits > 24)
     return fail(SONG_EUNSUPPORTED, "bloom_log2_bits %d outside [0, 24]", p->bloom_log2_bits);
   if (p->warps_per_block < 0 || p->warps_per_block > SONG_LB_THREADS / 32)
     return fail(SONG_EINVAL, "warps_per_block %d outside [0, %d]", p->warps_per_block, SONG_LB_THREADS / 32);
   if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
-  if (p->reserved != 0) return fail(SONG_EINVAL, "reserved must be 0");
   return SONG_OK;
 }
 
@@ -275,8 +235,18 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.L = p->queue_len;
   a.cosine = ix->metric == SONG_COSINE;
   a.dedup = ix->dedup;
-  const bool bloom = p->visited == SONG_VISITED_BLOOM;
-  Shape sh = search_shape(p->queue_len, bloom, p->bloom_log2_bits, ix->dpad);
+  int vk = song::VK_HASH;
+  a.sel = 1;
+  switch (p->visited) {
+    case SONG_VISITED_BLOOM: vk = song::VK_BLOOM; break;
+    case SONG_VISITED_HASH_GLOBAL: vk = song::VK_GHASH; a.sel = 0; break;
+    case SONG_VISITED_HASH_GLOBAL_SEL: vk = song::VK_GHASH; break;
+    case SONG_VISITED_CUCKOO: vk = song::VK_CUCKOO; break;
+    default: break;
+  }
+  a.gtab = nullptr;
+  a.gen0 = 0;
+  Shape sh = search_shape(p->queue_len, vk, p, ix->dpad);
   a.table_log2 = sh.table_log2;
   a.rebuild_at = sh.rebuild_at;
   a.warp_smem_bytes = sh.warp_bytes;
@@ -291,10 +261,10 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   ix->last_stream = st;
   const int m = ix->metric, qr = sh.qr, bps = p->blocks_per_sm, sms = ix->num_sms;
   switch (sh.nch) {
-    case 1: return launch_m<1>(a, m, bloom, qr, warps, bps, sms, st);
-    case 2: return launch_m<2>(a, m, bloom, qr, warps, bps, sms, st);
-    case 4: return launch_m<4>(a, m, bloom, qr, warps, bps, sms, st);
-    default: return launch_m<8>(a, m, bloom, qr, warps, bps, sms, st);
+    case 1: return launch_m<1>(ix, a, m, vk, qr, warps, bps, sms, st);
+    case 2: return launch_m<2>(ix, a, m, vk, qr, warps, bps, sms, st);
+    case 4: return launch_m<4>(ix, a, m, vk, qr, warps, bps, sms, st);
+    default: return launch_m<8>(ix, a, m, vk, qr, warps, bps, sms, st);
   }
 }
 
@@ -455,6 +425,9 @@ int song_index_last_status(song_index* ix) {
   CUDA_TRY(cudaMemset(ix->d_status, 0, sizeof st));
   if (st & song::STATUS_BAD_INPUT) return fail(SONG_EINVAL, "a query had a non-finite value");
   if (st & song::STATUS_ITER_CAP) return fail(SONG_EITERCAP, "a query reached max_iters");
+  if (st & song::STATUS_TABLE_FULL)
+    return fail(SONG_EUNSUPPORTED, "a query filled half of its global visited table; raise "
+                                   "table_log2");
   return SONG_OK;
 }
 

@@ -1,0 +1,46 @@
+// song_internal.h — definitions shared by the library's translation units
+// (song_api.cu and launch_nch<N>.cu).  Not part of the public ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+
+#include "search_kernel.cuh"
+#include "song.h"
+
+struct song_index {
+  int device = 0;
+  int num_sms = 0;
+  int64_t n = 0;
+  int dim = 0, dpad = 0, degree = 0, metric = 0;
+  float* d_data = nullptr;
+  int32_t* d_adj = nullptr;
+  unsigned* d_ticket = nullptr;
+  int* d_status = nullptr;
+  int dedup = 1;                       // some adjacency row repeats an id
+  uint64_t* d_gtab = nullptr;          // global visited tables (HASH_GLOBAL kinds)
+  size_t gtab_bytes = 0;
+  uint64_t gen_next = 1;               // next generation base for d_gtab
+  cudaStream_t stream = nullptr;       // owned; used by song_search
+  cudaStream_t last_stream = nullptr;  // stream of the last search
+  // scratch for the host-buffer entry point
+  float* d_q = nullptr;
+  int32_t* d_ids = nullptr;
+  float* d_dists = nullptr;
+  size_t cap_q = 0, cap_out = 0;
+};
+
+namespace song {
+int fail(int code, const char* fmt, ...);
+}  // namespace song
+
+#define CUDA_TRY(expr)                                                                  \
+  do {                                                                                  \
+    cudaError_t e_ = (expr);                                                            \
+    if (e_ != cudaSuccess)                                                              \
+      return song::fail(e_ == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA,     \
+                        "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__,     \
+                        __LINE__);                                                      \
+  } while (0)

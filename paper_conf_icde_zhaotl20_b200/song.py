@@ -21,8 +21,10 @@ LIB_PATH = os.environ.get("SONG_LIB", os.path.join(_PKG, "libsong.so"))
 
 L2, IP, COSINE = 0, 1, 2
 METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
-VISITED_HASH, VISITED_BLOOM = 0, 1
-VISITED = {"hash": VISITED_HASH, "bloom": VISITED_BLOOM}
+VISITED_HASH, VISITED_BLOOM, VISITED_HASH_GLOBAL, VISITED_HASH_GLOBAL_SEL, VISITED_CUCKOO = range(5)
+# names follow the paper's Fig. 7 legend
+VISITED = {"hash": VISITED_HASH, "bloom": VISITED_BLOOM, "hashtable": VISITED_HASH_GLOBAL,
+           "hashtable-sel": VISITED_HASH_GLOBAL_SEL, "cuckoo": VISITED_CUCKOO}
 
 STATUS = {0: "SONG_OK", -1: "SONG_EINVAL", -2: "SONG_ENOMEM", -3: "SONG_ECUDA",
           -4: "SONG_EUNSUPPORTED", -5: "SONG_EITERCAP"}
@@ -43,7 +45,7 @@ class SearchParams(ctypes.Structure):
                 ("visited", ctypes.c_int32), ("bloom_log2_bits", ctypes.c_int32),
                 ("entry", ctypes.c_int32), ("max_iters", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
-                ("id_offset", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -123,6 +125,7 @@ class Params:
     warps_per_block: int = 0
     blocks_per_sm: int = 0
     id_offset: int = 0
+    table_log2: int = 0
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -134,6 +137,7 @@ class Params:
         p.warps_per_block = self.warps_per_block
         p.blocks_per_sm = self.blocks_per_sm
         p.id_offset = self.id_offset
+        p.table_log2 = self.table_log2
         return p
 
 

@@ -26,21 +26,31 @@ def song():
     return s
 
 
-ORACLE_FLAGS = {"hash": oracle.OPTIMIZED, "bloom": oracle.OPTIMIZED_BLOOM}
+ORACLE_FLAGS = {"hash": oracle.OPTIMIZED, "bloom": oracle.OPTIMIZED_BLOOM,
+                "hashtable": oracle.HASHTABLE, "hashtable-sel": oracle.HASHTABLE_SEL,
+                "cuckoo": oracle.OPTIMIZED_CUCKOO}
+ALL_VISITED = list(ORACLE_FLAGS)
 
 
-def gpu_search(idx, q, K, L, visited="hash", **kw):
+def gpu_search(idx, q, K, L, visited="hash", allow_cap=False, **kw):
     s = song()
     p = s.Params(K=K, queue_len=L, visited=visited, **kw)
     qt = torch.as_tensor(q, device="cuda")
     ids, d, c = idx.search(qt, params=p, counters=True)
     torch.cuda.synchronize()
-    idx.last_status()
+    try:
+        idx.last_status()
+    except s.SongError as e:
+        if not (allow_cap and e.code == -5):
+            raise
     return ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy()
 
 
-def bloom_bits_for(L, log2=0):
-    return (1 << log2) if log2 else oracle.default_bloom_bits(L)
+def bloom_bits_for(L, log2=0, visited="bloom"):
+    """The oracle's filter size for a GPU run: Bloom bits or Cuckoo buckets."""
+    if log2:
+        return 1 << log2
+    return oracle.default_cuckoo_buckets(L) if visited == "cuckoo" else oracle.default_bloom_bits(L)
 
 
 def assert_exact(g, o):
@@ -63,7 +73,7 @@ def assert_close(g, o, truth=None, id_frac=0.995, scale=1.0):
 
 
 # ---------------------------------------------------------------- toy / P1-P2
-@pytest.mark.parametrize("visited", ["hash", "bloom"])
+@pytest.mark.parametrize("visited", ALL_VISITED)
 def test_fig1_toy_on_gpu(visited):
     data, adj, _, result = pins.load_toy()
     s = song()
@@ -73,7 +83,7 @@ def test_fig1_toy_on_gpu(visited):
     if visited == "hash":
         assert c[0].tolist() == [12, 4]  # Fig. 4(c): 12 distances, 4 expansions
     o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
-                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(3))
+                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(3, visited=visited))
     assert_exact((ids, d, c), o)
 
 
@@ -89,14 +99,14 @@ def tiny():
 
 
 @pytest.mark.parametrize("L", [10, 64, 257])
-@pytest.mark.parametrize("visited", ["hash", "bloom"])
+@pytest.mark.parametrize("visited", ALL_VISITED)
 def test_tiny_parity(tiny, L, visited):
     cfg, x, q, adj, truth = tiny
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q, cfg.K, L, visited)
     o = oracle.search(x, adj, q, cfg.K, L, flags=ORACLE_FLAGS[visited],
-                      bloom_bits=bloom_bits_for(L))
+                      bloom_bits=bloom_bits_for(L, visited=visited))
     assert_close(g, o, truth, scale=float(np.abs(o[1]).max()))
 
 
@@ -111,15 +121,44 @@ def sift100k():
 
 @pytest.mark.parametrize("L,visited,warps", [(10, "hash", 4), (16, "hash", 1), (64, "hash", 4),
                                             (200, "hash", 3), (64, "bloom", 4),
-                                            (1024, "hash", 2)])
+                                            (1024, "hash", 2), (48, "hashtable", 4),
+                                            (48, "hashtable-sel", 2), (48, "cuckoo", 4),
+                                            (300, "cuckoo", 2), (300, "hashtable-sel", 4)])
 def test_sift_integer_bit_exact(sift100k, L, visited, warps):
     cfg, x, q, adj = sift100k
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q.cpu().numpy(), cfg.K, L, visited, warps_per_block=warps)
     o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, L,
-                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L), nthreads=8)
+                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L, visited=visited),
+                      nthreads=8)
     assert_exact(g, o)
+
+
+def test_sift_small_cuckoo_filter_exact(sift100k):
+    """A 16/64-bucket Cuckoo filter overflows constantly: kicks, drops,
+    fingerprint collisions and the false negatives they cause (re-admitted
+    vertices) must follow the oracle's order exactly.  A lossy filter
+    can make the search revisit forever, so both sides cap expansions."""
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    for L in (24, 160):
+        for tl in (4, 6):
+            g = gpu_search(idx, q.cpu().numpy(), cfg.K, L, "cuckoo", allow_cap=True,
+                           table_log2=tl, max_iters=3000)
+            o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, L,
+                              flags=oracle.OPTIMIZED_CUCKOO, bloom_bits=1 << tl, nthreads=8,
+                              max_iters=3000)
+            assert_exact(g, o)
+
+
+def test_global_table_full_is_reported(sift100k):
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    with pytest.raises(s.SongError, match="EUNSUPPORTED"):
+        gpu_search(idx, q.cpu().numpy()[:32], cfg.K, 64, "hashtable", table_log2=6)
 
 
 def test_sift_small_bloom_filter_exact(sift100k):
@@ -178,17 +217,17 @@ def small_random(n=3000, dim=30, deg=12, seed=0, integer=True):
 
 
 @pytest.mark.parametrize("dim", [1, 3, 30, 130, 257])
-@pytest.mark.parametrize("L,K", [(1, 1), (7, 7), (33, 10), (100, 100)])
+@pytest.mark.parametrize("L,K", [(1, 1), (7, 7), (33, 10), (100, 100), (150, 20)])
 def test_edges_exact(dim, L, K):
     """ragged dims (row padding), degree < 32 with -1 padding and repeats,
     L = K = 1 (greedy), K = L, queue sizes that are not multiples of 32."""
     x, adj, q = small_random(dim=dim)
     s = song()
     idx = s.SongIndex(x, adj)
-    for visited in ("hash", "bloom"):
+    for visited in ALL_VISITED:
         g = gpu_search(idx, q, K, L, visited)
         o = oracle.search(x, adj, q, K, L, flags=ORACLE_FLAGS[visited],
-                          bloom_bits=bloom_bits_for(L))
+                          bloom_bits=bloom_bits_for(L, visited=visited))
         assert_exact(g, o)
 
 
