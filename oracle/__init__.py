@@ -6,7 +6,7 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R10 it follows are listed in its header and in DESIGN.md §3).
+R1-R12 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
@@ -25,8 +25,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "song_oracle.cpp")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
-L2, IP, COSINE = 0, 1, 2
-METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
+L2, IP, COSINE, HAMMING = 0, 1, 2, 3
+METRICS = {"l2": L2, "ip": IP, "cosine": COSINE, "hamming": HAMMING}
 
 # Mode flags (must match song_oracle.cpp's enum Flags).
 PLAIN = 0
@@ -78,6 +78,9 @@ def _load():
         lib.oracle_cuckoo_probe.restype = ctypes.c_int64
         lib.oracle_cuckoo_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
                                             ctypes.c_int64, P]
+        lib.oracle_rp_encode.restype = None
+        lib.oracle_rp_encode.argtypes = [P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, P,
+                                         ctypes.c_int32]
         lib.oracle_bloom_probe.restype = None
         lib.oracle_bloom_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
                                            ctypes.c_int64, P]
@@ -186,6 +189,51 @@ def bloom_probe(bits: int, inserted, probes):
     out = np.empty(pr.shape[0], np.uint8)
     lib.oracle_bloom_probe(int(bits), _ptr(ins), ins.shape[0], _ptr(pr), pr.shape[0], _ptr(out))
     return out.astype(bool)
+
+
+def rp_encode(data, R, nthreads: int = 1):
+    """1-bit random projection (§VII; reading R11): codes [n, h/32]
+    uint32, bit j = [<x, r_j> > 0] accumulated in fp64, LSB-first packing.
+    ``R`` is [h, dim] (row j = r_j); h % 32 == 0."""
+    lib = _load()
+    data = _f32(data)
+    R = _f32(R)
+    n, dim = data.shape
+    h = R.shape[0]
+    assert R.shape[1] == dim and h % 32 == 0 and h > 0
+    codes = np.empty((n, h // 32), np.uint32)
+    lib.oracle_rp_encode(_ptr(data), n, dim, _ptr(R), h, _ptr(codes), int(nthreads))
+    return codes
+
+
+def _codes_as_f32(codes):
+    c = np.ascontiguousarray(codes, dtype=np.uint32)
+    if c.ndim == 1:
+        c = c[None, :]
+    return c.view(np.float32)
+
+
+def search_codes(codes, adj, qcodes, K: int, L: int, flags: int = OPTIMIZED, **kw):
+    """Algorithm 1 over h-bit codes with the Hamming distance (reading R12).
+    codes [n, h/32] / qcodes [nq, h/32] uint32; returns as :func:`search`."""
+    return search(_codes_as_f32(codes), adj, _codes_as_f32(qcodes), K, L, metric=HAMMING,
+                  flags=flags, **kw)
+
+
+def bruteforce_codes(codes, qcodes, K: int, nthreads: int = 1):
+    """Exact top-K under (Hamming distance, id)."""
+    return bruteforce(_codes_as_f32(codes), _codes_as_f32(qcodes), K, metric=HAMMING,
+                      nthreads=nthreads)
+
+
+def hamming(a, b) -> int:
+    """Hamming distance of two codes through the oracle's R12 routine."""
+    return int(distance(_codes_as_f32(a)[0], _codes_as_f32(b)[0], HAMMING))
+
+
+def code_bytes(n: int, h: int) -> int:
+    """Table IV: an h-bit code takes h/32 words = h/8 bytes per point."""
+    return n * h // 8
 
 
 def recall(found_ids, truth_ids) -> float:

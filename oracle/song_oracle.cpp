@@ -33,6 +33,16 @@
 //      per-candidate interleaving for exact visited sets; fixes the operation
 //      order for the probabilistic filters).
 //   R10 Cuckoo filter: see struct Cuckoo.
+//   R11 1-bit random projection (§VII): bit j of a point's code is
+//      1 iff <x, r_j> > 0 (sgn(0) -> bit 0), the projection accumulated in fp64
+//      in dimension order; bit j lives in 32-bit word j / 32 at bit position
+//      j % 32 ("h can be set as a multiple of 32 so that the bit vector can be
+//      stored as several 32-bit unsigned integers").  R is [h][dim].
+//   R12 Hamming search: the distance of two codes is the number of differing
+//      bits ("the hamming distance between the bit-vectors"), used as the
+//      key's distance (an integer, exact in fp32) with the same (dist, id)
+//      order; the graph is the one built on the original vectors (the
+//      index is kept, only the dataset is reduced).
 //
 // Parity status: every function below is pinned by tests/test_oracle_*.py
 // (Fig. 1 / Fig. 4(c) traces, plain == optimized equivalence, brute-force
@@ -50,7 +60,7 @@
 
 namespace {
 
-enum Metric { ORACLE_L2 = 0, ORACLE_IP = 1, ORACLE_COSINE = 2 };
+enum Metric { ORACLE_L2 = 0, ORACLE_IP = 1, ORACLE_COSINE = 2, ORACLE_HAMMING = 3 };
 
 // Mode flags.  ORACLE_PLAIN (= 0) is Algorithm 1 literally: unbounded q,
 // exact visited set never deleted from, topk bounded at L (R1).
@@ -74,8 +84,23 @@ bool operator<(const Key& a, const Key& b) {
   return a.id < b.id;
 }
 
+// R12: Hamming distance of two h-bit codes stored as dim = h / 32 words (the
+// float pointers carry the code words bit for bit); bits counted one by one.
+float hamming(const float* p, const float* x, int words) {
+  int64_t diff = 0;
+  for (int i = 0; i < words; ++i) {
+    uint32_t a, b;
+    std::memcpy(&a, p + i, 4);
+    std::memcpy(&b, x + i, 4);
+    const uint32_t d = a ^ b;
+    for (int bit = 0; bit < 32; ++bit) diff += (d >> bit) & 1u;
+  }
+  return (float)diff;
+}
+
 // R7: the distance of §VI, accumulated in fp64 in index order.
 float distance(const float* p, const float* x, int dim, int metric) {
+  if (metric == ORACLE_HAMMING) return hamming(p, x, dim);
   double out;
   if (metric == ORACLE_L2) {
     double acc = 0.0;
@@ -424,6 +449,33 @@ void oracle_bruteforce(const float* data, int64_t n, int32_t dim, int32_t metric
   for (int t = 0; t < nthreads; ++t)
     pool.emplace_back([&, t]() {
       for (int64_t i = t; i < nq; i += nthreads) one(i);
+    });
+  for (auto& th : pool) th.join();
+}
+
+// 1-bit random projection of §VII (R11): codes[i] = the h-bit code
+// of data[i], packed in h / 32 uint32 words.  R is [h][dim] row-major (row j =
+// the random vector r_j).  h must be a multiple of 32.
+void oracle_rp_encode(const float* data, int64_t n, int32_t dim, const float* R, int32_t h,
+                      uint32_t* codes, int32_t nthreads) {
+  const int words = h / 32;
+  auto one = [&](int64_t i) {
+    const float* x = data + i * dim;
+    for (int w = 0; w < words; ++w) codes[i * words + w] = 0u;
+    for (int j = 0; j < h; ++j) {
+      double acc = 0.0;
+      for (int t = 0; t < dim; ++t) acc += (double)x[t] * (double)R[(int64_t)j * dim + t];
+      if (acc > 0.0) codes[i * words + j / 32] |= 1u << (j % 32);
+    }
+  };
+  if (nthreads <= 1) {
+    for (int64_t i = 0; i < n; ++i) one(i);
+    return;
+  }
+  std::vector<std::thread> pool;
+  for (int t = 0; t < nthreads; ++t)
+    pool.emplace_back([&, t]() {
+      for (int64_t i = t; i < n; i += nthreads) one(i);
     });
   for (auto& th : pool) th.join();
 }

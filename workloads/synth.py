@@ -37,6 +37,12 @@ CONFIGS = {
     "gist1m": Config("gist1m", 1_000_000, 960, "l2", 32, 1_000, 10, 200, "gist"),
     "glove200": Config("glove200", 1_183_514, 200, "ip", 32, 10_000, 10, 300, "glove"),
     "nytimes256": Config("nytimes256", 289_761, 256, "cosine", 32, 10_000, 10, 400, "nytimes"),
+    # §VII / Fig. 14: MNIST8m and its 1M sample, searched top-1 through
+    # 1-bit random-projection codes of h bits (extra["hash_bits"])
+    "mnist1m": Config("mnist1m", 1_000_000, 784, "l2", 32, 10_000, 1, 600, "mnist",
+                      extra={"hash_bits": 128}),
+    "mnist8m": Config("mnist8m", 8_090_000, 784, "l2", 32, 10_000, 1, 600, "mnist",
+                      extra={"hash_bits": 128}),
 }
 
 
@@ -141,6 +147,74 @@ class ClusteredSkewed:
         return out
 
 
+class MnistLike:
+    """MNIST8m-shaped (Table I; "less skewness"): 28 x 28 images,
+    integer pixels in [0, 255], ~20 % non-zero.  10 classes x 20 prototypes, each
+    the sum of 3-5 soft strokes (segments with a Gaussian profile); a sample is
+    a prototype under a random shift of up to +-2 px, an intensity jitter and
+    pixel noise on the ink, thresholded, scaled to 255 and rounded."""
+
+    SIDE = 28
+    PROTOS = 200
+    SHIFT = 2
+
+    def __init__(self, dim: int, seed: int, device="cpu"):
+        assert dim == self.SIDE * self.SIDE
+        g = _gen(seed * 7919 + 17, device)
+        self.dim, self.device = dim, device
+        S = self.SIDE
+        yy, xx = torch.meshgrid(torch.arange(S, device=device, dtype=torch.float32),
+                                torch.arange(S, device=device, dtype=torch.float32), indexing="ij")
+        protos = torch.zeros(self.PROTOS, S, S, device=device)
+        nstroke = torch.randint(3, 6, (self.PROTOS,), generator=g, device=device)
+        ends = 5.0 + 18.0 * torch.rand(self.PROTOS, 5, 2, 2, generator=g, device=device)
+        for s in range(5):
+            a, b = ends[:, s, 0], ends[:, s, 1]                      # [P, 2] (y, x)
+            ab = b - a
+            t = ((yy[None] - a[:, 0, None, None]) * ab[:, 0, None, None] +
+                 (xx[None] - a[:, 1, None, None]) * ab[:, 1, None, None])
+            t = (t / (ab * ab).sum(1).clamp_min(1e-6)[:, None, None]).clamp(0, 1)
+            py = a[:, 0, None, None] + t * ab[:, 0, None, None]
+            px = a[:, 1, None, None] + t * ab[:, 1, None, None]
+            d2 = (yy[None] - py) ** 2 + (xx[None] - px) ** 2
+            ink = torch.exp(-d2 / (2 * 1.35 ** 2))
+            protos += ink * (s < nstroke).float()[:, None, None]
+        protos = protos / protos.amax(dim=(1, 2), keepdim=True)
+        # every shifted copy of every prototype, flattened: [P * 25, 784]
+        pad = torch.nn.functional.pad(protos, (self.SHIFT,) * 4)
+        views = []
+        for dy in range(2 * self.SHIFT + 1):
+            for dx in range(2 * self.SHIFT + 1):
+                views.append(pad[:, dy:dy + S, dx:dx + S])
+        self.base = torch.stack(views, 1).reshape(-1, dim)
+
+    def sample(self, m: int, seed: int) -> torch.Tensor:
+        g = _gen(seed, self.device)
+        out = torch.empty(m, self.dim, device=self.device)
+        step = 1 << 16
+        nb = self.base.shape[0]
+        for s in range(0, m, step):
+            k = min(step, m - s)
+            b = self.base[torch.randint(0, nb, (k,), generator=g, device=self.device)]
+            gain = 0.8 + 0.4 * torch.rand(k, 1, generator=g, device=self.device)
+            x = b * gain + 0.08 * torch.randn(k, self.dim, generator=g, device=self.device) * (b > 0.1)
+            x = torch.where(x > 0.25, x, torch.zeros_like(x))
+            out[s:s + k] = torch.clamp(torch.round(x * 255.0), 0, 255)
+        return out
+
+
+def rp_matrix(h: int, dim: int, seed: int, device="cpu") -> torch.Tensor:
+    """The random vectors r_1..r_h of §VII's 1-bit random projection (P:467:
+    "entries ... iid standard normal"), [h, dim].  Drawn N(0, 1), then rounded
+    to multiples of 1/64 and clipped to [-4, 4]: every projection of integer
+    pixels is then an exact multiple of 1/64 far below 2^24 / 64, so its sign
+    (the code bit) is the same in fp32 in any summation order and in the
+    oracle's fp64 (tests check the bound).  Passed to both sides as an input."""
+    g = _gen(seed, device)
+    r = torch.randn(h, dim, generator=g, device=device, dtype=torch.float32)
+    return torch.clamp(torch.round(r * 64.0), -256, 256) / 64.0
+
+
 def generator_for(cfg: Config, device="cpu"):
     if cfg.kind == "sift":
         return SiftLike(cfg.dim, cfg.seed, device)
@@ -150,6 +224,8 @@ def generator_for(cfg: Config, device="cpu"):
         return ClusteredSkewed(cfg.dim, cfg.seed, 2000, False, device)
     if cfg.kind == "nytimes":
         return ClusteredSkewed(cfg.dim, cfg.seed, 500, True, device)
+    if cfg.kind == "mnist":
+        return MnistLike(cfg.dim, cfg.seed, device)
     return None
 
 
