@@ -40,7 +40,11 @@ extern "C" {
 
 typedef struct song_index song_index; /* opaque; owns its device copies */
 
-typedef enum { SONG_L2 = 0, SONG_IP = 1, SONG_COSINE = 2 } song_metric;
+/* SONG_HAMMING: the index holds h-bit codes of the 1-bit random projection
+ * (§VII) and the distance is the Hamming distance (number of
+ * differing bits, returned as an exact integer-valued float).  Such indexes
+ * are made only by song_index_create_codes / song_index_create_rp. */
+typedef enum { SONG_L2 = 0, SONG_IP = 1, SONG_COSINE = 2, SONG_HAMMING = 3 } song_metric;
 
 typedef enum {
   SONG_OK = 0,
@@ -73,6 +77,7 @@ typedef enum {
 #define SONG_MAX_DEGREE 32
 #define SONG_MAX_DIM 1024
 #define SONG_MAX_QUEUE_LEN 2048
+#define SONG_MAX_CODE_BITS 1024
 
 typedef struct song_search_params {
   int32_t K;               /* results per query, 1 <= K <= queue_len */
@@ -104,6 +109,12 @@ typedef struct song_index_info {
   int64_t graph_bytes;     /* n * degree * 4 (Table III) */
   int32_t device;          /* CUDA device ordinal */
   int32_t num_sms;         /* SMs on that device */
+  int32_t code_bits;       /* SONG_HAMMING: h bits per code (dim_padded is then the
+                              row stride in 32-bit words, vector_bytes the codes'
+                              bytes, Table IV, and dim the length of the float
+                              queries song_search accepts: the original dimension for
+                              an index made by song_index_create_rp, else 0); else 0 */
+  int32_t reserved;        /* 0 (keeps the struct free of implicit padding) */
 } song_index_info;
 
 /* Fill p with the library defaults for (K, queue_len). Never fails. */
@@ -169,6 +180,51 @@ int song_index_last_status(song_index* idx);
 int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,
                     int32_t Kin, int32_t K, int32_t* ids_out, float* dists_out,
                     void* stream);
+
+/* ---- 1-bit random projection (§VII "Out-of-GPU-memory datasets") ----
+ * "For two data vectors u, v ... we generate a random vector r with entries in
+ * iid standard normal ... With h independent random vectors, each data point
+ * is mapped into an h-bit vector. The hamming distance between the
+ * bit-vectors becomes an good estimate of the similarity".
+ * Code layout (reading R11): bit j = [<x, r_j> > 0] (a zero
+ * projection gives 0), stored in 32-bit word j / 32 at bit j % 32; a code is
+ * h / 32 words ("h can be set as a multiple of 32").  R is [h][dim]
+ * fp32 row-major (row j = r_j), drawn by the caller. */
+
+/* Encode n DEVICE vectors [n][dim] fp32 with DEVICE R [bits][dim] into DEVICE
+ * codes [n][bits/32] uint32 (dense rows).  fp32 accumulation; asynchronous on
+ * stream.  Errors: SONG_EINVAL (NULL, n < 1, dim < 1, bits not a positive
+ * multiple of 32), SONG_EUNSUPPORTED (bits > SONG_MAX_CODE_BITS), SONG_ECUDA. */
+int song_rp_encode(const float* vectors, int64_t n, int32_t dim, const float* R, int32_t bits,
+                   uint32_t* codes, void* stream);
+
+/* Create a SONG_HAMMING index from HOST codes [n][bits/32] uint32 and HOST
+ * adjacency [n][degree] int32 (both copied).  Queries then go through
+ * song_search_codes_ex.  Errors as song_index_create, plus SONG_EINVAL for
+ * bits not a positive multiple of 32, SONG_EUNSUPPORTED for bits >
+ * SONG_MAX_CODE_BITS. */
+int song_index_create_codes(const uint32_t* codes, int64_t n, int32_t bits,
+                            const int32_t* adjacency, int32_t degree, song_index** out);
+
+/* Create a SONG_HAMMING index from HOST vectors [n][dim] fp32 that need not fit
+ * in device memory: the vectors are streamed to the device in chunks,
+ * encoded with HOST R [bits][dim] (copied; kept by the index) and only the
+ * codes stay resident.  adjacency is HOST [n][degree] int32 (the graph built on
+ * the original vectors).  song_search / song_search_ex then take float
+ * queries [nq][dim], encoded on the device with the same R before the search.
+ * Errors as song_index_create_codes, plus SONG_EINVAL for a non-finite vector
+ * or R value. */
+int song_index_create_rp(const float* vectors, int64_t n, int32_t dim, const float* R,
+                         int32_t bits, const int32_t* adjacency, int32_t degree,
+                         song_index** out);
+
+/* Search a SONG_HAMMING index with DEVICE query codes [nq][bits/32] uint32;
+ * otherwise as song_search_ex (same params, outputs, counters and errors;
+ * params.visited must be SONG_VISITED_HASH or SONG_VISITED_BLOOM, else
+ * SONG_EUNSUPPORTED).  Returned distances are Hamming distances. */
+int song_search_codes_ex(song_index* idx, const song_search_params* params,
+                         const uint32_t* query_codes, int64_t nq, int32_t* ids_out,
+                         float* dists_out, int32_t* counters_out, void* stream);
 
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);

@@ -82,6 +82,12 @@ template <int NCH>
 int launch_m(song_index* ix, const SearchArgs& a, int metric, int vk, int qr, int warps,
              int bps, int sms, cudaStream_t st) {
   if (metric == SONG_L2) return launch_v<NCH, MET_L2>(ix, a, vk, qr, warps, bps, sms, st);
+  if (metric == SONG_HAMMING) {
+    // codes: the two shared-memory visited sets of §IV (hash-sel-del, Bloom)
+    if (vk == VK_BLOOM) return launch_q<NCH, MET_HAM, VK_BLOOM>(ix, a, qr, warps, bps, sms, st);
+    if (vk == VK_HASH) return launch_q<NCH, MET_HAM, VK_HASH>(ix, a, qr, warps, bps, sms, st);
+    return fail(SONG_EUNSUPPORTED, "Hamming indexes support the hash and Bloom visited sets");
+  }
   return launch_v<NCH, MET_DOT>(ix, a, vk, qr, warps, bps, sms, st);
 }
 

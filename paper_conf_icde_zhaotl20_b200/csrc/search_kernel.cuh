@@ -44,12 +44,14 @@ constexpr int STAGE_BYTES = 16384;  // per-warp row stage (32 rows of d = 128)
 enum : int { STATUS_BAD_INPUT = 1, STATUS_ITER_CAP = 2, STATUS_TABLE_FULL = 4 };
 // visited-set kinds (template parameter VK of the kernel)
 enum : int { VK_HASH = 0, VK_BLOOM = 1, VK_GHASH = 2, VK_CUCKOO = 3 };
-enum : int { MET_L2 = 0, MET_DOT = 1 };
+// MET_HAM: rows are h-bit codes of the 1-bit random projection (§VII),
+// dpad 32-bit words each; the distance is the Hamming distance (reading R12)
+enum : int { MET_L2 = 0, MET_DOT = 1, MET_HAM = 2 };
 
 struct SearchArgs {
-  const float* data;      // [n][dpad], 16 B aligned rows
+  const float* data;      // [n][dpad], 16 B aligned rows (MET_HAM: uint32 code words)
   const int32_t* adj;     // [n][degree]
-  const float* queries;   // [nq][dim] (caller layout, unpadded)
+  const float* queries;   // [nq][dim] (caller layout, unpadded; MET_HAM: [nq][dim] words)
   int32_t* ids_out;       // [nq][K]
   float* dists_out;       // [nq][K]
   int32_t* counters_out;  // [nq][2] or nullptr
@@ -651,10 +653,34 @@ __device__ __forceinline__ void zero_stage(float* stage, int rows, int lane) {
   __syncwarp();
 }
 
+// Hamming distance (§VII; reading R12): a code is dpad <= 4*NCH words,
+// so lane j gathers candidate j's whole code with NCH 16 B loads — all the
+// warp's rows in flight at once, no staging and no cross-lane reduction — and
+// XOR-popcounts it against the query code every lane holds in qv.
+template <int NCH>
+__device__ __forceinline__ float hamming_distance(const float* __restrict__ data, int dpad,
+                                                  const int* cid, int nc,
+                                                  const float4 (&qv)[NCH], int lane) {
+  int d = 0;
+  if (lane < nc) {
+    const uint4* row = reinterpret_cast<const uint4*>(data + (int64_t)cid[lane] * dpad);
+    uint4 v[NCH];
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      v[c] = (4 * c < dpad) ? __ldg(row + c) : make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      d += __popc(v[c].x ^ __float_as_uint(qv[c].x)) + __popc(v[c].y ^ __float_as_uint(qv[c].y)) +
+           __popc(v[c].z ^ __float_as_uint(qv[c].z)) + __popc(v[c].w ^ __float_as_uint(qv[c].w));
+  }
+  return (float)d;  // exact: d <= 32 * dpad < 2^24
+}
+
 template <int NCH, int METRIC>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
                                                float* stage, int cosine, int lane) {
+  if constexpr (METRIC == MET_HAM) return hamming_distance<NCH>(data, dpad, cid, nc, qv, lane);
   constexpr int R = StageRows<NCH>::R;
   constexpr int NBUF = StageRows<NCH>::NBUF;
   constexpr int LR = Log2<R>::value;
@@ -744,7 +770,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   const int L = a.L;
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
   float* stage = reinterpret_cast<float*>(base);                       // staged rows
-  const size_t stage_bytes = (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
+  const size_t stage_bytes =  // (Hamming codes are gathered straight into registers)
+      METRIC == MET_HAM ? 0 : (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
   int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
@@ -764,7 +791,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
   GHash gh{a.gtab + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2),
            a.table_log2, a.gen0};
   const unsigned lt = lanemask_lt();
-  zero_stage<NCH>(stage, StageRows<NCH>::NBUF * R, lane);
+  if (METRIC != MET_HAM) zero_stage<NCH>(stage, StageRows<NCH>::NBUF * R, lane);
 
   // ---- visited-set operations (§IV-B/D/E) for the four kinds
   auto v_contains = [&](int v, bool act) -> bool {
@@ -811,6 +838,16 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_k
     float4 qv[NCH];
     bool bad = false;
     const float* qrow = a.queries + (int64_t)qi * a.dim;
+    if constexpr (METRIC == MET_HAM) {
+      // every lane holds the whole query code (words 4c .. 4c+3 in qv[c]);
+      // words past dim are 0, like the index's padding words
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) {
+        const int e = 4 * c;
+        qv[c] = make_float4(e + 0 < a.dim ? qrow[e + 0] : 0.f, e + 1 < a.dim ? qrow[e + 1] : 0.f,
+                            e + 2 < a.dim ? qrow[e + 2] : 0.f, e + 3 < a.dim ? qrow[e + 3] : 0.f);
+      }
+    } else
 #pragma unroll
     for (int c = 0; c < NCH; ++c) {
       int e = (c * 32 + lane) * 4;

@@ -9,10 +9,12 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
 #include "merge_kernel.cuh"
+#include "rp_kernel.cuh"
 #include "search_kernel.cuh"
 #include "song.h"
 
@@ -128,6 +130,8 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_ids);
   cudaFree(ix->d_dists);
   cudaFree(ix->d_gtab);
+  cudaFree(ix->d_R);
+  cudaFree(ix->d_qcodes);
   if (ix->stream) cudaStreamDestroy(ix->stream);
   delete ix;
 }
@@ -139,7 +143,10 @@ int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* a
   if (!vectors || !adjacency) return fail(SONG_EINVAL, "vectors/adjacency is NULL");
   if (n < 1 || dim < 1 || degree < 1) return fail(SONG_EINVAL, "n, dim and degree must be >= 1");
   if (n > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n must fit int32 ids");
-  if (metric < SONG_L2 || metric > SONG_COSINE) return fail(SONG_EINVAL, "unknown metric %d", (int)metric);
+  if (metric < SONG_L2 || metric > SONG_COSINE)
+    return fail(SONG_EINVAL, "metric %d: float indexes take SONG_L2, SONG_IP or SONG_COSINE "
+                             "(SONG_HAMMING indexes come from song_index_create_codes/_rp)",
+                (int)metric);
   if (degree > SONG_MAX_DEGREE) return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
   if (dim > SONG_MAX_DIM) return fail(SONG_EUNSUPPORTED, "dim %d > %d", dim, SONG_MAX_DIM);
   return SONG_OK;
@@ -160,7 +167,7 @@ struct Shape {
   int nch;
 };
 
-Shape search_shape(int L, int vk, const song_search_params* p, int dpad) {
+Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
   Shape s;
   int tbytes = 0;
   s.rebuild_at = 0;
@@ -185,11 +192,13 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad) {
     s.rebuild_at = big ? (3 << s.table_log2) / 4 : (SONG_HASH_REBUILD_NUM << s.table_log2) / 16;
     tbytes = (1 << s.table_log2) * 4;
   }
-  s.nch = (dpad + 127) / 128;
+  // float rows: NCH = 16 B chunks per lane (128 floats per chunk row);
+  // Hamming codes: NCH = 16 B chunks per code (4 words), no row stage
+  s.nch = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
   const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
-  const int stage_bytes = SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE rows
+  const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   s.warp_bytes = stage_bytes + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
@@ -246,7 +255,9 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   }
   a.gtab = nullptr;
   a.gen0 = 0;
-  Shape sh = search_shape(p->queue_len, vk, p, ix->dpad);
+  if (ix->metric == SONG_HAMMING && vk != song::VK_HASH && vk != song::VK_BLOOM)
+    return fail(SONG_EUNSUPPORTED, "Hamming indexes support the hash and Bloom visited sets");
+  Shape sh = search_shape(p->queue_len, vk, p, ix->dpad, ix->metric == SONG_HAMMING);
   a.table_log2 = sh.table_log2;
   a.rebuild_at = sh.rebuild_at;
   a.warp_smem_bytes = sh.warp_bytes;
@@ -292,9 +303,199 @@ int finish_create(song_index* ix, cudaStream_t st) {
   return SONG_OK;
 }
 
+int check_bits(int32_t bits) {
+  if (bits < 32 || bits % 32) return fail(SONG_EINVAL, "bits %d is not a positive multiple of 32", bits);
+  if (bits > SONG_MAX_CODE_BITS) return fail(SONG_EUNSUPPORTED, "bits %d > %d", bits, SONG_MAX_CODE_BITS);
+  return SONG_OK;
+}
+
+// §VII encoder launch: X [n][ldx] -> codes [n][ldc] words (first bits/32 used)
+int launch_rp(const float* X, int64_t n, int dim, int64_t ldx, const float* R, int bits,
+              uint32_t* codes, int64_t ldc, cudaStream_t st) {
+  const int64_t tiles = (n + song::RP_TM - 1) / song::RP_TM;
+  if (tiles > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n too large for one encode launch");
+  dim3 grid((unsigned)tiles, (unsigned)((bits + song::RP_TN - 1) / song::RP_TN));
+  song::rp_encode_kernel<<<grid, song::RP_THREADS, 0, st>>>(X, n, dim, ldx, R, bits, codes, ldc);
+  CUDA_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+// encode a float query batch of a song_index_create_rp index into ix->d_qcodes
+int encode_queries(song_index* ix, const float* q, int64_t nq, cudaStream_t st) {
+  const size_t need = (size_t)nq * ix->dim * sizeof(uint32_t);
+  if (need > ix->cap_qcodes) {
+    CUDA_TRY(cudaStreamSynchronize(st));
+    cudaFree(ix->d_qcodes);
+    ix->d_qcodes = nullptr;
+    ix->cap_qcodes = 0;
+    CUDA_TRY(cudaMalloc(&ix->d_qcodes, need));
+    ix->cap_qcodes = need;
+  }
+  return launch_rp(q, nq, ix->rp_dim, ix->rp_dim, ix->d_R, ix->code_bits, ix->d_qcodes, ix->dim,
+                   st);
+}
+
+int check_adjacency_host(const int32_t* adjacency, int64_t n, int32_t degree) {
+  for (int64_t i = 0; i < n * (int64_t)degree; ++i)
+    if (adjacency[i] < -1 || adjacency[i] >= n)
+      return fail(SONG_EINVAL, "adjacency[%lld] = %d outside [-1, %lld)", (long long)i,
+                  adjacency[i], (long long)n);
+  return SONG_OK;
+}
+
+// common part of the two SONG_HAMMING creators: a zeroed [n][dpad]-word code
+// array (padding words stay 0 on both sides of every XOR) and the adjacency
+int alloc_codes_index(int64_t n, int32_t bits, const int32_t* adjacency, int32_t degree,
+                      song_index** out, song_index** made) {
+  if (!out) return fail(SONG_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!adjacency) return fail(SONG_EINVAL, "adjacency is NULL");
+  if (n < 1 || degree < 1) return fail(SONG_EINVAL, "n and degree must be >= 1");
+  if (n > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n must fit int32 ids");
+  if (degree > SONG_MAX_DEGREE) return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
+  int rc = check_bits(bits);
+  if (rc) return rc;
+  rc = check_adjacency_host(adjacency, n, degree);
+  if (rc) return rc;
+  song_index* ix = new song_index();
+  rc = alloc_index(ix, n, bits / 32, degree, SONG_HAMMING);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  ix->code_bits = bits;
+  cudaError_t e = cudaMemsetAsync(ix->d_data, 0, (size_t)n * ix->dpad * 4, ix->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(ix->d_adj, adjacency, (size_t)n * degree * sizeof(int32_t),
+                        cudaMemcpyHostToDevice, ix->stream);
+  if (e != cudaSuccess) {
+    free_index(ix);
+    return fail(SONG_ECUDA, "index upload: %s", cudaGetErrorString(e));
+  }
+  *made = ix;
+  return SONG_OK;
+}
+
 }  // namespace
 
 extern "C" {
+
+int song_rp_encode(const float* vectors, int64_t n, int32_t dim, const float* R, int32_t bits,
+                   uint32_t* codes, void* stream) {
+  if (!vectors || !R || !codes) return fail(SONG_EINVAL, "NULL argument");
+  if (n < 1 || dim < 1) return fail(SONG_EINVAL, "n and dim must be >= 1");
+  int rc = check_bits(bits);
+  if (rc) return rc;
+  return launch_rp(vectors, n, dim, dim, R, bits, codes, bits / 32, (cudaStream_t)stream);
+}
+
+int song_index_create_codes(const uint32_t* codes, int64_t n, int32_t bits,
+                            const int32_t* adjacency, int32_t degree, song_index** out) {
+  if (!codes) {
+    if (out) *out = nullptr;
+    return fail(SONG_EINVAL, "codes is NULL");
+  }
+  song_index* ix = nullptr;
+  int rc = alloc_codes_index(n, bits, adjacency, degree, out, &ix);
+  if (rc) return rc;
+  const int words = bits / 32;
+  cudaError_t e = cudaMemcpy2DAsync(ix->d_data, ix->dpad * 4, codes, words * 4, words * 4, n,
+                                    cudaMemcpyHostToDevice, ix->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(ix->stream);
+  if (e != cudaSuccess) {
+    free_index(ix);
+    return fail(SONG_ECUDA, "codes upload: %s", cudaGetErrorString(e));
+  }
+  ix->dedup = 1;
+  rc = finish_create(ix, ix->stream);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  *out = ix;
+  return SONG_OK;
+}
+
+int song_index_create_rp(const float* vectors, int64_t n, int32_t dim, const float* R,
+                         int32_t bits, const int32_t* adjacency, int32_t degree,
+                         song_index** out) {
+  if (!vectors || !R) {
+    if (out) *out = nullptr;
+    return fail(SONG_EINVAL, "vectors/R is NULL");
+  }
+  if (dim < 1) return fail(SONG_EINVAL, "dim must be >= 1");
+  if (bits >= 32 && bits % 32 == 0)
+    for (int64_t i = 0; i < (int64_t)bits * dim; ++i)
+      if (!std::isfinite(R[i])) return fail(SONG_EINVAL, "R[%lld] is not finite", (long long)i);
+  song_index* ix = nullptr;
+  int rc = alloc_codes_index(n, bits, adjacency, degree, out, &ix);
+  if (rc) return rc;
+  ix->rp_dim = dim;
+  cudaStream_t st = ix->stream;
+  // the vectors need not fit in device memory — stream them through a
+  // double-buffered device chunk (<= 256 MiB each) and keep only the codes
+  int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(n, (256ll << 20) / (4ll * dim)));
+  if (const char* env = std::getenv("SONG_RP_CHUNK_ROWS"))  // tests: force many chunks
+    chunk = std::max<int64_t>(1, std::min<int64_t>(chunk, std::atoll(env)));
+  float* d_chunk[2] = {nullptr, nullptr};
+  unsigned long long* d_bad = nullptr;
+  cudaEvent_t done[2] = {nullptr, nullptr};
+  auto cleanup = [&]() {
+    cudaStreamSynchronize(st);
+    cudaFree(d_chunk[0]);
+    cudaFree(d_chunk[1]);
+    cudaFree(d_bad);
+    if (done[0]) cudaEventDestroy(done[0]);
+    if (done[1]) cudaEventDestroy(done[1]);
+  };
+  cudaError_t e = cudaMalloc(&ix->d_R, (size_t)bits * dim * 4);
+  if (e == cudaSuccess) e = cudaMalloc(&d_chunk[0], (size_t)chunk * dim * 4);
+  if (e == cudaSuccess && chunk < n) e = cudaMalloc(&d_chunk[1], (size_t)chunk * dim * 4);
+  if (e == cudaSuccess) e = cudaMalloc(&d_bad, sizeof *d_bad);
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_bad, 0, sizeof *d_bad, st);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done[0], cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done[1], cudaEventDisableTiming);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(ix->d_R, R, (size_t)bits * dim * 4, cudaMemcpyHostToDevice, st);
+  for (int64_t s0 = 0, k = 0; e == cudaSuccess && s0 < n; s0 += chunk, ++k) {
+    const int64_t rows = std::min(chunk, n - s0);
+    float* buf = d_chunk[k & 1];
+    e = cudaEventSynchronize(done[k & 1]);  // the encode that last read buf is finished
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(buf, vectors + s0 * dim, (size_t)rows * dim * 4, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) break;
+    validate_kernel<<<592, 256, 0, st>>>(buf, rows * dim, nullptr, 0, n, d_bad);
+    rc = launch_rp(buf, rows, dim, dim, ix->d_R, bits,
+                   reinterpret_cast<uint32_t*>(ix->d_data) + s0 * ix->dpad, ix->dpad, st);
+    if (rc) {
+      cleanup();
+      free_index(ix);
+      return rc;
+    }
+    e = cudaEventRecord(done[k & 1], st);
+  }
+  unsigned long long bad = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&bad, d_bad, sizeof bad, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  cleanup();
+  if (e != cudaSuccess) {
+    free_index(ix);
+    return fail(e == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA, "rp index: %s",
+                cudaGetErrorString(e));
+  }
+  if (bad) {
+    free_index(ix);
+    return fail(SONG_EINVAL, "%llu non-finite vector values", bad);
+  }
+  rc = finish_create(ix, st);
+  if (rc) {
+    free_index(ix);
+    return rc;
+  }
+  *out = ix;
+  return SONG_OK;
+}
+
 
 void song_default_params(song_search_params* p, int32_t K, int32_t queue_len) {
   if (!p) return;
@@ -403,6 +604,9 @@ int song_index_get_info(const song_index* ix, song_index_info* info) {
   info->graph_bytes = ix->n * (int64_t)ix->degree * 4;
   info->device = ix->device;
   info->num_sms = ix->num_sms;
+  info->code_bits = ix->code_bits;
+  info->reserved = 0;
+  if (ix->metric == SONG_HAMMING) info->dim = ix->rp_dim;
   return SONG_OK;
 }
 
@@ -413,8 +617,28 @@ int song_search_ex(song_index* ix, const song_search_params* p, const float* que
   if (nq > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "nq must fit int32");
   int rc = check_params(ix, p);
   if (rc) return rc;
+  if (ix->metric == SONG_HAMMING) {
+    if (!ix->d_R)
+      return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
+    rc = encode_queries(ix, queries, nq, (cudaStream_t)stream);
+    if (rc) return rc;
+    queries = reinterpret_cast<const float*>(ix->d_qcodes);
+  }
   return enqueue_search(ix, p, queries, nq, ids_out, dists_out, counters_out,
                         (cudaStream_t)stream);
+}
+
+int song_search_codes_ex(song_index* ix, const song_search_params* p, const uint32_t* qcodes,
+                         int64_t nq, int32_t* ids_out, float* dists_out, int32_t* counters_out,
+                         void* stream) {
+  if (!ix || !p || !qcodes || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (ix->metric != SONG_HAMMING) return fail(SONG_EINVAL, "not a SONG_HAMMING index");
+  if (nq < 1) return fail(SONG_EINVAL, "nq must be >= 1");
+  if (nq > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "nq must fit int32");
+  int rc = check_params(ix, p);
+  if (rc) return rc;
+  return enqueue_search(ix, p, reinterpret_cast<const float*>(qcodes), nq, ids_out, dists_out,
+                        counters_out, (cudaStream_t)stream);
 }
 
 int song_index_last_status(song_index* ix) {
@@ -439,7 +663,10 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
   song_default_params(&p, K, queue_len);
   int rc = check_params(ix, &p);
   if (rc) return rc;
-  const size_t qbytes = (size_t)nq * ix->dim * sizeof(float);
+  if (ix->metric == SONG_HAMMING && !ix->d_R)
+    return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
+  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
+  const size_t qbytes = (size_t)nq * qdim * sizeof(float);
   const size_t obytes = (size_t)nq * K * sizeof(int32_t);
   if (qbytes > ix->cap_q) {
     cudaFree(ix->d_q);
@@ -460,7 +687,13 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
   }
   cudaStream_t st = ix->stream;
   CUDA_TRY(cudaMemcpyAsync(ix->d_q, queries, qbytes, cudaMemcpyHostToDevice, st));
-  rc = enqueue_search(ix, &p, ix->d_q, nq, ix->d_ids, ix->d_dists, nullptr, st);
+  const float* dq = ix->d_q;
+  if (ix->metric == SONG_HAMMING) {
+    rc = encode_queries(ix, ix->d_q, nq, st);
+    if (rc) return rc;
+    dq = reinterpret_cast<const float*>(ix->d_qcodes);
+  }
+  rc = enqueue_search(ix, &p, dq, nq, ix->d_ids, ix->d_dists, nullptr, st);
   if (rc) return rc;
   CUDA_TRY(cudaMemcpyAsync(ids_out, ix->d_ids, obytes, cudaMemcpyDeviceToHost, st));
   CUDA_TRY(cudaMemcpyAsync(dists_out, ix->d_dists, obytes, cudaMemcpyDeviceToHost, st));

@@ -30,6 +30,12 @@ struct song_index {
   int32_t* d_ids = nullptr;
   float* d_dists = nullptr;
   size_t cap_q = 0, cap_out = 0;
+  // SONG_HAMMING (§VII): dim / dpad count 32-bit code words
+  int code_bits = 0;
+  int rp_dim = 0;                      // length of float queries (0: codes only)
+  float* d_R = nullptr;                // [code_bits][rp_dim] random vectors
+  uint32_t* d_qcodes = nullptr;        // scratch: encoded query batch
+  size_t cap_qcodes = 0;
 };
 
 namespace song {

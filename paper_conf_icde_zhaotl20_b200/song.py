@@ -19,8 +19,8 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SONG_LIB", os.path.join(_PKG, "libsong.so"))
 
-L2, IP, COSINE = 0, 1, 2
-METRICS = {"l2": L2, "ip": IP, "cosine": COSINE}
+L2, IP, COSINE, HAMMING = 0, 1, 2, 3
+METRICS = {"l2": L2, "ip": IP, "cosine": COSINE, "hamming": HAMMING}
 VISITED_HASH, VISITED_BLOOM, VISITED_HASH_GLOBAL, VISITED_HASH_GLOBAL_SEL, VISITED_CUCKOO = range(5)
 # names follow the paper's Fig. 7 legend
 VISITED = {"hash": VISITED_HASH, "bloom": VISITED_BLOOM, "hashtable": VISITED_HASH_GLOBAL,
@@ -31,7 +31,9 @@ STATUS = {0: "SONG_OK", -1: "SONG_EINVAL", -2: "SONG_ENOMEM", -3: "SONG_ECUDA",
 
 EXPORTED = ["song_default_params", "song_index_create", "song_index_create_device",
             "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
-            "song_index_last_status", "song_merge_topk", "song_last_error", "song_version"]
+            "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
+            "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
+            "song_search_codes_ex"]
 
 
 class SongError(RuntimeError):
@@ -52,7 +54,8 @@ class IndexInfo(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("dim", ctypes.c_int32), ("dim_padded", ctypes.c_int32),
                 ("degree", ctypes.c_int32), ("metric", ctypes.c_int32),
                 ("vector_bytes", ctypes.c_int64), ("graph_bytes", ctypes.c_int64),
-                ("device", ctypes.c_int32), ("num_sms", ctypes.c_int32)]
+                ("device", ctypes.c_int32), ("num_sms", ctypes.c_int32),
+                ("code_bits", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 _lib = None
@@ -78,13 +81,19 @@ def lib():
         L.song_search_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
         L.song_index_last_status.argtypes = [P]
         L.song_merge_topk.argtypes = [P, P, i32, i64, i32, i32, P, P, P]
+        L.song_rp_encode.argtypes = [P, i64, i32, P, i32, P, P]
+        L.song_index_create_codes.argtypes = [P, i64, i32, P, i32, PP]
+        L.song_index_create_rp.argtypes = [P, i64, i32, P, i32, P, i32, PP]
+        L.song_search_codes_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
         L.song_version.argtypes = []
         for name in ("song_index_create", "song_index_create_device", "song_index_destroy",
                      "song_index_get_info", "song_search", "song_search_ex",
-                     "song_index_last_status", "song_merge_topk"):
+                     "song_index_last_status", "song_merge_topk", "song_rp_encode",
+                     "song_index_create_codes", "song_index_create_rp",
+                     "song_search_codes_ex"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -147,10 +156,18 @@ class SongIndex:
     ``vectors`` [n, dim] float32 and ``adjacency`` [n, degree] int32 may be
     numpy arrays (host create) or CUDA tensors (device create)."""
 
-    def __init__(self, vectors, adjacency, metric: str = "l2"):
+    def __init__(self, vectors, adjacency, metric: str = "l2", *, _handle=None):
         self._h = ctypes.c_void_p()
         self.metric = metric
+        if _handle is not None:  # made by from_codes / from_rp
+            self._h = _handle
+            self.device = None
+            info = self.info()
+            self.n, self.dim, self.degree = info.n, info.dim, info.degree
+            self.code_bits = info.code_bits
+            return
         m = METRICS[metric]
+        self.code_bits = 0
         if _is_cuda_tensor(vectors):
             torch = _torch()
             v = vectors.contiguous().to(torch.float32)
@@ -171,6 +188,50 @@ class SongIndex:
                 a.ctypes.data_as(ctypes.c_void_p), a.shape[1], m, ctypes.byref(self._h)))
         info = self.info()
         self.n, self.dim, self.degree = info.n, info.dim, info.degree
+
+    @classmethod
+    def from_codes(cls, codes: np.ndarray, bits: int, adjacency) -> "SongIndex":
+        """song_index_create_codes: HOST codes [n, bits/32] uint32 (§VII)."""
+        c = np.ascontiguousarray(codes, np.uint32)
+        a = np.ascontiguousarray(adjacency, np.int32)
+        h = ctypes.c_void_p()
+        _check(lib().song_index_create_codes(c.ctypes.data_as(ctypes.c_void_p), c.shape[0], bits,
+                                             a.ctypes.data_as(ctypes.c_void_p), a.shape[1],
+                                             ctypes.byref(h)))
+        return cls(None, None, "hamming", _handle=h)
+
+    @classmethod
+    def from_rp(cls, vectors: np.ndarray, R: np.ndarray, adjacency) -> "SongIndex":
+        """song_index_create_rp: HOST vectors [n, dim] streamed to the device and
+        encoded with HOST R [bits, dim]; only the codes stay resident."""
+        v = np.ascontiguousarray(vectors, np.float32)
+        r = np.ascontiguousarray(R, np.float32)
+        a = np.ascontiguousarray(adjacency, np.int32)
+        assert r.shape[1] == v.shape[1]
+        h = ctypes.c_void_p()
+        _check(lib().song_index_create_rp(v.ctypes.data_as(ctypes.c_void_p), v.shape[0],
+                                          v.shape[1], r.ctypes.data_as(ctypes.c_void_p),
+                                          r.shape[0], a.ctypes.data_as(ctypes.c_void_p),
+                                          a.shape[1], ctypes.byref(h)))
+        return cls(None, None, "hamming", _handle=h)
+
+    def search_codes(self, qcodes, params: "Params", counters: bool = False):
+        """song_search_codes_ex on CUDA uint32/int32 code tensors [nq, bits/32]."""
+        torch = _torch()
+        if not _is_cuda_tensor(qcodes):
+            raise TypeError("search_codes() takes a CUDA tensor")
+        q = qcodes.contiguous()
+        assert q.element_size() == 4
+        nq = q.shape[0]
+        ids = torch.empty((nq, params.K), dtype=torch.int32, device=q.device)
+        dists = torch.empty((nq, params.K), dtype=torch.float32, device=q.device)
+        ctr = torch.empty((nq, 2), dtype=torch.int32, device=q.device) if counters else None
+        cp = params.to_c()
+        _check(lib().song_search_codes_ex(
+            self._h, ctypes.byref(cp), ctypes.c_void_p(q.data_ptr()), nq,
+            ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(dists.data_ptr()),
+            ctypes.c_void_p(ctr.data_ptr() if ctr is not None else 0), _stream_ptr(q.device)))
+        return (ids, dists, ctr) if counters else (ids, dists)
 
     def info(self) -> IndexInfo:
         inf = IndexInfo()
@@ -248,6 +309,21 @@ def merge_topk(ids, dists, K: int):
                                  G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
                                  ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
     return oi, od
+
+
+def rp_encode(vectors, R):
+    """song_rp_encode: CUDA tensors vectors [n, dim], R [bits, dim] fp32 ->
+    codes [n, bits/32] (int32 tensor holding the uint32 words, §VII)."""
+    torch = _torch()
+    v = vectors.contiguous().float()
+    r = R.to(device=v.device, dtype=torch.float32).contiguous()
+    bits = r.shape[0]
+    codes = torch.empty((v.shape[0], bits // 32 if bits % 32 == 0 else 1), dtype=torch.int32,
+                        device=v.device)
+    _check(lib().song_rp_encode(ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1],
+                                ctypes.c_void_p(r.data_ptr()), bits,
+                                ctypes.c_void_p(codes.data_ptr()), _stream_ptr(v.device)))
+    return codes
 
 
 def version() -> str:

@@ -55,10 +55,24 @@ def test_argument_errors_need_no_gpu():
     assert (p.K, p.queue_len, p.visited, p.entry, p.id_offset) == (10, 64, 0, 0, 0)
 
 
-def test_params_struct_layout_matches_header():
+def test_params_struct_layout_matches_header(tmp_path):
+    """The ctypes mirrors have the C compiler's sizes and field offsets."""
+    import subprocess
     from paper_conf_icde_zhaotl20_b200 import song
-    assert ctypes.sizeof(song.SearchParams) == 40
-    assert ctypes.sizeof(song.IndexInfo) == 48
+    src = tmp_path / "layout.c"
+    src.write_text(
+        '#include <stdio.h>\n#include <stddef.h>\n#include "song.h"\n'
+        'int main(void){printf("%zu %zu %zu %zu %zu\\n", sizeof(song_search_params),'
+        ' sizeof(song_index_info), offsetof(song_index_info, vector_bytes),'
+        ' offsetof(song_index_info, code_bits), offsetof(song_search_params, table_log2));'
+        'return 0;}\n')
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(src),
+                           "-o", str(exe)])
+    c = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
+    assert c == [ctypes.sizeof(song.SearchParams), ctypes.sizeof(song.IndexInfo),
+                 song.IndexInfo.vector_bytes.offset, song.IndexInfo.code_bits.offset,
+                 song.SearchParams.table_log2.offset]
 
 
 def test_product_package_does_not_import_oracle():
@@ -69,3 +83,30 @@ def test_product_package_does_not_import_oracle():
                 text = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in text and "from oracle" not in text, f
                 assert "song_oracle" not in text and "liboracle" not in text, f
+
+
+def test_rp_argument_errors_need_no_gpu():
+    """§VII entry points validate before any CUDA call."""
+    import numpy as np
+    from paper_conf_icde_zhaotl20_b200 import song
+    lib = song.lib()
+    out = ctypes.c_void_p()
+    codes = np.zeros((4, 2), np.uint32)
+    adj = np.zeros((4, 2), np.int32)
+    P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+    assert lib.song_rp_encode(None, 4, 8, None, 64, None, None) == -1
+    # bits must be a positive multiple of 32, at most SONG_MAX_CODE_BITS
+    assert lib.song_index_create_codes(P(codes), 4, 48, P(adj), 2, ctypes.byref(out)) == -1
+    assert lib.song_index_create_codes(P(codes), 4, 0, P(adj), 2, ctypes.byref(out)) == -1
+    assert lib.song_index_create_codes(P(codes), 4, 2048, P(adj), 2, ctypes.byref(out)) == -4
+    assert lib.song_index_create_codes(None, 4, 64, P(adj), 2, ctypes.byref(out)) == -1
+    bad = adj.copy()
+    bad[1, 1] = 4  # id out of range
+    assert lib.song_index_create_codes(P(codes), 4, 64, P(bad), 2, ctypes.byref(out)) == -1
+    assert not out.value
+    # float creators reject SONG_HAMMING
+    v = np.zeros((4, 8), np.float32)
+    assert lib.song_index_create(P(v), 4, 8, P(adj), 2, 3, ctypes.byref(out)) == -1
+    R = np.zeros((64, 8), np.float32)
+    R[0, 0] = np.nan
+    assert lib.song_index_create_rp(P(v), 4, 8, P(R), 64, P(adj), 2, ctypes.byref(out)) == -1
