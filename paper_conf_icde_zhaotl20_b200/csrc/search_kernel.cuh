@@ -653,7 +653,8 @@ __device__ __forceinline__ void zero_stage(float* stage, int rows, int lane) {
   __syncwarp();
 }
 
-// Hamming distance (§VII; reading R12): a code is dpad <= 4*NCH words,
+// Hamming distance (§VII; reading R12): a code is dpad <= 4*NCH words
+// (dpad = 1, 2 or a multiple of 4),
 // so lane j gathers candidate j's whole code with NCH 16 B loads — all the
 // warp's rows in flight at once, no staging and no cross-lane reduction — and
 // XOR-popcounts it against the query code every lane holds in qv.
@@ -662,7 +663,17 @@ __device__ __forceinline__ float hamming_distance(const float* __restrict__ data
                                                   const int* cid, int nc,
                                                   const float4 (&qv)[NCH], int lane) {
   int d = 0;
-  if (lane < nc) {
+  if (dpad < 4) {  // 32- and 64-bit codes are stored unpadded (1 or 2 words)
+    if (lane < nc) {
+      const uint32_t* w = reinterpret_cast<const uint32_t*>(data) + (int64_t)cid[lane] * dpad;
+      if (dpad == 2) {
+        const uint2 v = __ldg(reinterpret_cast<const uint2*>(w));
+        d = __popc(v.x ^ __float_as_uint(qv[0].x)) + __popc(v.y ^ __float_as_uint(qv[0].y));
+      } else {
+        d = __popc(__ldg(w) ^ __float_as_uint(qv[0].x));
+      }
+    }
+  } else if (lane < nc) {
     const uint4* row = reinterpret_cast<const uint4*>(data + (int64_t)cid[lane] * dpad);
     uint4 v[NCH];
 #pragma unroll
@@ -760,8 +771,15 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
 #define SONG_LB_BLOCKS 6
 #endif
 // QR > 0: q / topk in registers (queue_len <= 32*QR); QR == 0: shared memory.
+// wide rows (NCH >= 4: d > 256 floats, or 512/1024-bit codes) hold 4-8 float4
+// of query per lane: give them 128 registers (4 CTAs/SM) instead of spilling
+template <int NCH>
+struct MinBlocks {
+  static constexpr int value = NCH >= 4 ? 4 : SONG_LB_BLOCKS;
+};
 template <int NCH, int METRIC, int VK, int QR>
-__global__ void __launch_bounds__(SONG_LB_THREADS, SONG_LB_BLOCKS) song_search_kernel(const SearchArgs a) {
+__global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
+    song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH>::R;
   constexpr bool DEL = (VK == VK_HASH || VK == VK_CUCKOO);  // visited deletion (§IV-E)

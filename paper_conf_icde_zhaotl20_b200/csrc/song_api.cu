@@ -107,7 +107,9 @@ int alloc_index(song_index* ix, int64_t n, int32_t dim, int32_t degree, song_met
   CUDA_TRY(cudaDeviceGetAttribute(&ix->num_sms, cudaDevAttrMultiProcessorCount, ix->device));
   ix->n = n;
   ix->dim = dim;
-  ix->dpad = (dim + 3) & ~3;
+  // float rows: 16 B multiples; codes: 1, 2 or a multiple of 4 words, so
+  // h = 32 / 64 take exactly h / 8 bytes per point (Table IV)
+  ix->dpad = (metric == SONG_HAMMING && (dim == 1 || dim == 2)) ? dim : (dim + 3) & ~3;
   ix->degree = degree;
   ix->metric = (int)metric;
   CUDA_TRY(cudaMalloc(&ix->d_data, (size_t)n * ix->dpad * sizeof(float)));

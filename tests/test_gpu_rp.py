@@ -101,7 +101,7 @@ def test_rp_index_end_to_end(mnist, monkeypatch, chunk_rows):
     idx = s.SongIndex.from_rp(x, R, adj)
     info = idx.info()
     assert (info.code_bits, info.dim, info.dim_padded, info.metric) == (128, 784, 4, 3)
-    assert info.vector_bytes == x.shape[0] * bits // 8  # Table IV's layout
+    assert info.vector_bytes == x.shape[0] * bits // 8  # Table IV layout
     ids, d, c = idx.search(torch.as_tensor(q, device="cuda"),
                            params=s.Params(K=1, queue_len=64), counters=True)
     torch.cuda.synchronize()
@@ -137,4 +137,29 @@ def test_hamming_errors(mnist):
     assert (d.cpu().numpy() == 0).all()
     oi, od, _, _ = oracle.search_codes(codes, adj, np.zeros((2, 4), np.uint32), 5, 16)
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
+    idx.close()
+
+
+@pytest.mark.parametrize("bits", [32, 64, 96, 128, 160, 256])
+def test_code_footprint_is_table4s(mnist, bits):
+    """Table IV: h/8 bytes per point (h = 96 / 160 round up to 16 B)."""
+    x, q, adj = mnist
+    R = rp_matrix(bits, 784, 603).numpy()
+    codes = oracle.rp_encode(x, R, nthreads=8)
+    qc = oracle.rp_encode(q[:50], R)
+    s = song()
+    idx = s.SongIndex.from_codes(codes, bits, adj)
+    info = idx.info()
+    words = bits // 32
+    padded = words if words <= 2 else (words + 3) // 4 * 4
+    assert info.vector_bytes == x.shape[0] * padded * 4
+    if bits in (32, 64, 128, 256):
+        assert info.vector_bytes == x.shape[0] * bits // 8
+    ids, d, c = idx.search_codes(torch.as_tensor(qc.view(np.int32), device="cuda"),
+                                 s.Params(K=5, queue_len=40), counters=True)
+    torch.cuda.synchronize()
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 5, 40)
+    np.testing.assert_array_equal(ids.cpu().numpy(), oi)
+    np.testing.assert_array_equal(d.cpu().numpy(), od)
+    np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
     idx.close()

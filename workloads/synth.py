@@ -149,55 +149,65 @@ class ClusteredSkewed:
 
 class MnistLike:
     """MNIST8m-shaped (Table I; "less skewness"): 28 x 28 images,
-    integer pixels in [0, 255], ~20 % non-zero.  10 classes x 20 prototypes, each
-    the sum of 3-5 soft strokes (segments with a Gaussian profile); a sample is
-    a prototype under a random shift of up to +-2 px, an intensity jitter and
-    pixel noise on the ink, thresholded, scaled to 255 and rounded."""
+    integer pixels in [0, 255], ~20 % non-zero, every sample distinct (MNIST8m
+    is MNIST under random deformations).  10 classes x 20 prototypes, each 3-5
+    strokes (segments); a sample takes a prototype, jitters every stroke end
+    (N(0, 1.2 px)), applies a random similarity transform (rotation +-0.25
+    rad, scale 0.85-1.15, shift +-2 px) and a random pen width (1.0-1.6 px),
+    renders the strokes with a Gaussian profile, applies an intensity gain,
+    thresholds, scales to 255 and rounds."""
 
     SIDE = 28
     PROTOS = 200
-    SHIFT = 2
+    STROKES = 5
 
     def __init__(self, dim: int, seed: int, device="cpu"):
         assert dim == self.SIDE * self.SIDE
         g = _gen(seed * 7919 + 17, device)
         self.dim, self.device = dim, device
+        self.nstroke = torch.randint(3, self.STROKES + 1, (self.PROTOS,), generator=g, device=device)
+        # stroke ends in a centred 18 x 18 box: [P, S, 2 ends, (y, x)]
+        self.ends = 5.0 + 18.0 * torch.rand(self.PROTOS, self.STROKES, 2, 2, generator=g,
+                                            device=device)
         S = self.SIDE
         yy, xx = torch.meshgrid(torch.arange(S, device=device, dtype=torch.float32),
                                 torch.arange(S, device=device, dtype=torch.float32), indexing="ij")
-        protos = torch.zeros(self.PROTOS, S, S, device=device)
-        nstroke = torch.randint(3, 6, (self.PROTOS,), generator=g, device=device)
-        ends = 5.0 + 18.0 * torch.rand(self.PROTOS, 5, 2, 2, generator=g, device=device)
-        for s in range(5):
-            a, b = ends[:, s, 0], ends[:, s, 1]                      # [P, 2] (y, x)
-            ab = b - a
-            t = ((yy[None] - a[:, 0, None, None]) * ab[:, 0, None, None] +
-                 (xx[None] - a[:, 1, None, None]) * ab[:, 1, None, None])
-            t = (t / (ab * ab).sum(1).clamp_min(1e-6)[:, None, None]).clamp(0, 1)
-            py = a[:, 0, None, None] + t * ab[:, 0, None, None]
-            px = a[:, 1, None, None] + t * ab[:, 1, None, None]
-            d2 = (yy[None] - py) ** 2 + (xx[None] - px) ** 2
-            ink = torch.exp(-d2 / (2 * 1.35 ** 2))
-            protos += ink * (s < nstroke).float()[:, None, None]
-        protos = protos / protos.amax(dim=(1, 2), keepdim=True)
-        # every shifted copy of every prototype, flattened: [P * 25, 784]
-        pad = torch.nn.functional.pad(protos, (self.SHIFT,) * 4)
-        views = []
-        for dy in range(2 * self.SHIFT + 1):
-            for dx in range(2 * self.SHIFT + 1):
-                views.append(pad[:, dy:dy + S, dx:dx + S])
-        self.base = torch.stack(views, 1).reshape(-1, dim)
+        self.grid = torch.stack([yy.reshape(-1), xx.reshape(-1)], 1)  # [784, 2]
+
+    def _render(self, ends, live, width):
+        """ends [k, S, 2, 2] pixel coords, live [k, S] bool, width [k] -> [k, 784] ink."""
+        a, b = ends[:, :, 0], ends[:, :, 1]                      # [k, S, 2]
+        ab = b - a
+        p = self.grid[None, None]                                # [1, 1, 784, 2]
+        t = ((p - a[:, :, None]) * ab[:, :, None]).sum(-1)
+        t = (t / (ab * ab).sum(-1).clamp_min(1e-6)[:, :, None]).clamp(0, 1)
+        near = a[:, :, None] + t[..., None] * ab[:, :, None]     # [k, S, 784, 2]
+        d2 = ((p - near) ** 2).sum(-1)                           # [k, S, 784]
+        ink = torch.exp(-d2 / (2 * width[:, None, None] ** 2)) * live[:, :, None]
+        return ink.amax(1)                                       # [k, 784]
 
     def sample(self, m: int, seed: int) -> torch.Tensor:
         g = _gen(seed, self.device)
-        out = torch.empty(m, self.dim, device=self.device)
-        step = 1 << 16
-        nb = self.base.shape[0]
+        dev = self.device
+        out = torch.empty(m, self.dim, device=dev)
+        step = 8192
+        c0 = (self.SIDE - 1) / 2.0
         for s in range(0, m, step):
             k = min(step, m - s)
-            b = self.base[torch.randint(0, nb, (k,), generator=g, device=self.device)]
-            gain = 0.8 + 0.4 * torch.rand(k, 1, generator=g, device=self.device)
-            x = b * gain + 0.08 * torch.randn(k, self.dim, generator=g, device=self.device) * (b > 0.1)
+            pid = torch.randint(0, self.PROTOS, (k,), generator=g, device=dev)
+            ends = self.ends[pid] + 1.2 * torch.randn(k, self.STROKES, 2, 2, generator=g, device=dev)
+            ang = (torch.rand(k, generator=g, device=dev) - 0.5) * 0.5
+            scl = 0.85 + 0.3 * torch.rand(k, generator=g, device=dev)
+            sh = (torch.rand(k, 2, generator=g, device=dev) - 0.5) * 4.0
+            cos, sin = torch.cos(ang) * scl, torch.sin(ang) * scl
+            rot = torch.stack([torch.stack([cos, -sin], 1), torch.stack([sin, cos], 1)], 1)
+            e = ends - c0
+            e = torch.einsum("kij,ksej->ksei", rot, e) + c0 + sh[:, None, None, :]
+            live = torch.arange(self.STROKES, device=dev)[None] < self.nstroke[pid][:, None]
+            width = 1.0 + 0.6 * torch.rand(k, generator=g, device=dev)
+            ink = self._render(e, live, width)
+            gain = 0.8 + 0.4 * torch.rand(k, 1, generator=g, device=dev)
+            x = ink * gain
             x = torch.where(x > 0.25, x, torch.zeros_like(x))
             out[s:s + k] = torch.clamp(torch.round(x * 255.0), 0, 255)
         return out
