@@ -6,7 +6,7 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R12 it follows are listed in its header and in DESIGN.md §3).
+R1-R13 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
@@ -70,6 +70,12 @@ def _load():
             P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
             ctypes.c_int64, ctypes.c_int32, ctypes.c_int64, P, P, P,
             ctypes.c_int32, _TRACE_FN, P]
+        lib.oracle_search_steps.restype = ctypes.c_int64
+        lib.oracle_search_steps.argtypes = [
+            P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, ctypes.c_int32,
+            P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+            ctypes.c_int64, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P,
+            ctypes.c_int32, _TRACE_FN, P]
         lib.oracle_distance.restype = ctypes.c_float
         lib.oracle_distance.argtypes = [P, P, ctypes.c_int32, ctypes.c_int32]
         lib.oracle_bruteforce.restype = None
@@ -125,10 +131,11 @@ def default_bloom_bits(L: int) -> int:
 
 def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OPTIMIZED,
            bloom_bits: Optional[int] = None, entry: int = 0, max_iters: int = 1 << 40,
-           nthreads: int = 1, trace: Optional[Callable] = None):
+           nthreads: int = 1, trace: Optional[Callable] = None, steps: int = 1):
     """Run the oracle.  Returns (ids [nq,K] int32, dists [nq,K] f32,
     counters [nq,2] int64 = (n_dist, n_exp), n_capped).  ``bloom_bits`` is the
-    Bloom filter's bit count, or the Cuckoo filter's bucket count."""
+    Bloom filter's bit count, or the Cuckoo filter's bucket count; ``steps`` is
+    the multi-step probing width (pops per iteration, reading R13)."""
     lib = _load()
     data = _f32(data)
     adj = _i32(adj)
@@ -153,9 +160,10 @@ def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OP
             v_ids = None if nv < 0 else [vp[i] for i in range(nv)]
             trace(int(it), q_ids, t_ids, v_ids)
         cb = _TRACE_FN(_cb)
-    capped = lib.oracle_search(_ptr(data), n, dim, _ptr(adj), degree, metric, _ptr(queries), nq,
-                               K, L, flags, int(bloom_bits), entry, int(max_iters), _ptr(ids),
-                               _ptr(dists), _ptr(counters), int(nthreads), cb, None)
+    capped = lib.oracle_search_steps(_ptr(data), n, dim, _ptr(adj), degree, metric,
+                                     _ptr(queries), nq, K, L, flags, int(bloom_bits), entry,
+                                     int(max_iters), int(steps), _ptr(ids), _ptr(dists),
+                                     _ptr(counters), int(nthreads), cb, None)
     return ids, dists, counters, int(capped)
 
 

@@ -38,6 +38,11 @@
 //      in dimension order; bit j lives in 32-bit word j / 32 at bit position
 //      j % 32 ("h can be set as a multiple of 32 so that the bit vector can be
 //      stored as several 32-bit unsigned integers").  R is [h][dim].
+//   R13 multi-step probing (§V): an iteration pops up to `steps` vertices
+//      (each checked against the termination rule with topk as updated by the
+//      previous pops), locates the unvisited neighbours of all of them into ONE
+//      candidate list (pop order, then row order, first occurrence), then runs
+//      the distance and maintenance stages once.  n_exp counts pops.
 //   R12 Hamming search: the distance of two codes is the number of differing
 //      bits ("the hamming distance between the bit-vectors"), used as the
 //      key's distance (an integer, exact in fp32) with the same (dist, id)
@@ -280,6 +285,7 @@ struct Problem {
   int K, L, flags, entry;
   uint64_t bloom_bits;  // Bloom: bits; Cuckoo: buckets
   int64_t max_iters;
+  int steps;            // multi-step probing: pops per iteration (R13), >= 1
 };
 
 // Algorithm 1 with the optimizations of §IV switched by flags.
@@ -306,6 +312,7 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
   emit_trace(cb, ctx, 0, q, topk, visited);
 
   std::vector<int32_t> cand;
+  std::vector<Key> popped;
   int64_t it = 0;
   // Step 2 — Alg. 1 line 2.
   while (!q.empty()) {
@@ -315,36 +322,47 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
     }
     ++it;
     // 2.1 — line 3: pop the minimum of q.
-    Key now = *q.begin();
-    q.erase(q.begin());
-    // 2.2 — lines 4-5: stop when topk is full and its max is better than now.
-    if ((int)topk.size() == L && *std::prev(topk.end()) < now) break;
-    // 2.3 — line 7 (+R1): push into topk; evict the max beyond L; [del] erase it
-    // from visited ("when the topk is updated, the popped-out vertex can
-    // also be deleted").
-    topk.insert(now);
-    if ((int)topk.size() > L) {
-      Key y = *std::prev(topk.end());
-      topk.erase(std::prev(topk.end()));
-      if (del) visited.erase(y.id);
+    // 2.1 / 2.2 / 2.3 for each of up to P.steps pops (multi-step probing, §V
+    // P:451, reading R13; steps = 1 is Alg. 1 exactly): pop the minimum of q
+    // (line 3); stop when topk is full and its max is better (lines 4-5) —
+    // before the first pop that ends the search, before a later pop that ends
+    // only this iteration's popping; push into topk, evict its max beyond L and
+    // [del] erase it from visited (line 7, R1).
+    popped.clear();
+    while ((int)popped.size() < P.steps && !q.empty()) {
+      Key now = *q.begin();
+      if ((int)topk.size() == L && *std::prev(topk.end()) < now) break;
+      q.erase(q.begin());
+      popped.push_back(now);
+      topk.insert(now);
+      if ((int)topk.size() > L) {
+        Key y = *std::prev(topk.end());
+        topk.erase(std::prev(topk.end()));
+        if (del) visited.erase(y.id);
+      }
     }
-    // 2.4 — candidate locating (§V): unvisited neighbours, row order,
-    // skipping padding and repeats (R6).
+    if (popped.empty()) break;
+    // 2.4 — candidate locating (§V): unvisited neighbours of the popped
+    // vertices, in pop order then row order, skipping padding and repeats (R6)
+    // — one candidate list for all pops ("fills more vertices into the
+    // candidate list").
     cand.clear();
-    const int32_t* row = P.adj + (int64_t)now.id * P.degree;
-    for (int j = 0; j < P.degree; ++j) {
-      int32_t v = row[j];
-      if (v < 0) continue;
-      if (visited.contains(v)) continue;
-      if (std::find(cand.begin(), cand.end(), v) != cand.end()) continue;
-      cand.push_back(v);
+    for (const Key& now : popped) {
+      const int32_t* row = P.adj + (int64_t)now.id * P.degree;
+      for (int j = 0; j < P.degree; ++j) {
+        int32_t v = row[j];
+        if (v < 0) continue;
+        if (visited.contains(v)) continue;
+        if (std::find(cand.begin(), cand.end(), v) != cand.end()) continue;
+        cand.push_back(v);
+      }
     }
     // 2.5 — bulk distance computation (§VI).
     std::vector<Key> ck;
     ck.reserve(cand.size());
     for (int32_t v : cand) ck.push_back(Key{distance(p, P.data + (int64_t)v * P.dim, P.dim, P.metric), v});
     n_dist += (int64_t)cand.size();
-    n_exp += 1;
+    n_exp += (int64_t)popped.size();
     // 2.6 — maintenance, lines 12-13 with §IV-C/D/E, as a batch (R9: "the data
     // structure maintenance stage uses the distances to update the priority
     // queues and the hash table"): insert the selected candidates in
@@ -387,17 +405,15 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
 
 extern "C" {
 
-// Search nq queries.  All pointers are host pointers; layouts are row-major:
-// data [n][dim] fp32, adj [n][degree] int32 (-1 = padding), queries [nq][dim],
-// ids/dists [nq][K], counters [nq][2] = (distance computations, expansions)
-// or NULL.  nthreads > 1 partitions the queries over std::threads (no trace).
-// Returns the number of queries that hit max_iters (0 = all finished).
-int64_t oracle_search(const float* data, int64_t n, int32_t dim, const int32_t* adj,
-                      int32_t degree, int32_t metric, const float* queries, int64_t nq,
-                      int32_t K, int32_t L, int32_t flags, int64_t bloom_bits, int32_t entry,
-                      int64_t max_iters, int32_t* ids, float* dists, int64_t* counters,
-                      int32_t nthreads, trace_fn cb, void* ctx) {
-  Problem P{data, n, dim, adj, degree, metric, K, L, flags, entry, (uint64_t)bloom_bits, max_iters};
+// As oracle_search, with `steps` pops per iteration (multi-step probing, R13).
+int64_t oracle_search_steps(const float* data, int64_t n, int32_t dim, const int32_t* adj,
+                            int32_t degree, int32_t metric, const float* queries, int64_t nq,
+                            int32_t K, int32_t L, int32_t flags, int64_t bloom_bits,
+                            int32_t entry, int64_t max_iters, int32_t steps, int32_t* ids,
+                            float* dists, int64_t* counters, int32_t nthreads, trace_fn cb,
+                            void* ctx) {
+  Problem P{data, n, dim, adj, degree, metric, K, L, flags, entry, (uint64_t)bloom_bits, max_iters,
+            steps < 1 ? 1 : steps};
   if (nthreads <= 1 || cb) {
     int64_t fails = 0;
     for (int64_t i = 0; i < nq; ++i)
@@ -418,6 +434,21 @@ int64_t oracle_search(const float* data, int64_t n, int32_t dim, const int32_t* 
   int64_t total = 0;
   for (int64_t f : fails) total += f;
   return total;
+}
+
+// Search nq queries.  All pointers are host pointers; layouts are row-major:
+// data [n][dim] fp32, adj [n][degree] int32 (-1 = padding), queries [nq][dim],
+// ids/dists [nq][K], counters [nq][2] = (distance computations, expansions)
+// or NULL.  nthreads > 1 partitions the queries over std::threads (no trace).
+// Returns the number of queries that hit max_iters (0 = all finished).
+int64_t oracle_search(const float* data, int64_t n, int32_t dim, const int32_t* adj,
+                      int32_t degree, int32_t metric, const float* queries, int64_t nq,
+                      int32_t K, int32_t L, int32_t flags, int64_t bloom_bits, int32_t entry,
+                      int64_t max_iters, int32_t* ids, float* dists, int64_t* counters,
+                      int32_t nthreads, trace_fn cb, void* ctx) {
+  return oracle_search_steps(data, n, dim, adj, degree, metric, queries, nq, K, L, flags,
+                             bloom_bits, entry, max_iters, 1, ids, dists, counters, nthreads, cb,
+                             ctx);
 }
 
 // The distance of §VI for one pair (exposed so tests can pin R7 directly).
