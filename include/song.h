@@ -78,6 +78,7 @@ typedef enum {
 #define SONG_MAX_DIM 1024
 #define SONG_MAX_QUEUE_LEN 2048
 #define SONG_MAX_CODE_BITS 1024
+#define SONG_MAX_STEPS 4
 
 typedef struct song_search_params {
   int32_t K;               /* results per query, 1 <= K <= queue_len */
@@ -97,6 +98,11 @@ typedef struct song_search_params {
                               query that fills half of it stops with SONG_EUNSUPPORTED
                               status; CUCKOO: log2 buckets of 4 (default: 4 slots per
                               live key bound 2L+32); ignored otherwise; 0 = default */
+  int32_t steps;           /* multi-step probing (§V, reading R13): up to
+                              `steps` vertices popped per iteration into one candidate
+                              list; 0 or 1 = Algorithm 1's single pop; at most
+                              SONG_MAX_STEPS; > 1 needs visited HASH or BLOOM and a
+                              float index (else SONG_EUNSUPPORTED) */
 } song_search_params;
 
 typedef struct song_index_info {

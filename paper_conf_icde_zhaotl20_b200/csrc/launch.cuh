@@ -33,10 +33,10 @@ inline int prepare_global_tables(song_index* ix, SearchArgs& a, int64_t warps_to
   return SONG_OK;
 }
 
-template <int NCH, int METRIC, int VK, int QR>
+template <int NCH, int METRIC, int VK, int QR, bool MS>
 int launch_t(song_index* ix, SearchArgs a, int warps, int blocks_per_sm, int num_sms,
              cudaStream_t st) {
-  auto kern = song_search_kernel<NCH, METRIC, VK, QR>;
+  auto kern = song_search_kernel<NCH, METRIC, VK, QR, MS>;
   const size_t smem = (size_t)a.warp_smem_bytes * warps;
   CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int fit = 0;
@@ -55,14 +55,14 @@ int launch_t(song_index* ix, SearchArgs a, int warps, int blocks_per_sm, int num
   return SONG_OK;
 }
 
-template <int NCH, int METRIC, int VK>
+template <int NCH, int METRIC, int VK, bool MS = false>
 int launch_q(song_index* ix, const SearchArgs& a, int qr, int warps, int bps, int sms,
              cudaStream_t st) {
   switch (qr) {
-    case 1: return launch_t<NCH, METRIC, VK, 1>(ix, a, warps, bps, sms, st);
-    case 2: return launch_t<NCH, METRIC, VK, 2>(ix, a, warps, bps, sms, st);
-    case 4: return launch_t<NCH, METRIC, VK, 4>(ix, a, warps, bps, sms, st);
-    default: return launch_t<NCH, METRIC, VK, 0>(ix, a, warps, bps, sms, st);
+    case 1: return launch_t<NCH, METRIC, VK, 1, MS>(ix, a, warps, bps, sms, st);
+    case 2: return launch_t<NCH, METRIC, VK, 2, MS>(ix, a, warps, bps, sms, st);
+    case 4: return launch_t<NCH, METRIC, VK, 4, MS>(ix, a, warps, bps, sms, st);
+    default: return launch_t<NCH, METRIC, VK, 0, MS>(ix, a, warps, bps, sms, st);
   }
 }
 
@@ -70,6 +70,12 @@ template <int NCH, int METRIC>
 int launch_v(song_index* ix, const SearchArgs& a, int vk, int qr, int warps, int bps,
              int sms, cudaStream_t st) {
   using namespace song;
+  // multi-step probing (a.steps > 1, §V): hash-sel-del and Bloom only
+  if (a.steps > 1) {
+    if (vk == VK_BLOOM) return launch_q<NCH, METRIC, VK_BLOOM, true>(ix, a, qr, warps, bps, sms, st);
+    if (vk == VK_HASH) return launch_q<NCH, METRIC, VK_HASH, true>(ix, a, qr, warps, bps, sms, st);
+    return fail(SONG_EUNSUPPORTED, "multi-step probing supports the hash and Bloom visited sets");
+  }
   switch (vk) {
     case VK_BLOOM: return launch_q<NCH, METRIC, VK_BLOOM>(ix, a, qr, warps, bps, sms, st);
     case VK_GHASH: return launch_q<NCH, METRIC, VK_GHASH>(ix, a, qr, warps, bps, sms, st);

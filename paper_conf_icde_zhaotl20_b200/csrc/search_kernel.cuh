@@ -63,6 +63,7 @@ struct SearchArgs {
   int K, L;
   int table_log2;  // hash: log2 slots; bloom: log2 bits
   int entry, max_iters, id_offset;
+  int steps;       // multi-step probing (§V, reading R13): pops per iteration
   int cosine;      // MET_DOT: 1 -> 1 - dot, 0 -> -dot
   int dedup;       // 1 if some adjacency row repeats an id
   int rebuild_at;  // hash: rebuild when live + tombstones would exceed this
@@ -777,7 +778,9 @@ template <int NCH>
 struct MinBlocks {
   static constexpr int value = NCH >= 4 ? 4 : SONG_LB_BLOCKS;
 };
-template <int NCH, int METRIC, int VK, int QR>
+// MS: multi-step probing (a.steps pops per iteration, <= MAX_STEPS; §V)
+constexpr int MAX_STEPS = 4;
+template <int NCH, int METRIC, int VK, int QR, bool MS = false>
 __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
     song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -791,7 +794,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
   const size_t stage_bytes =  // (Hamming codes are gathered straight into registers)
       METRIC == MET_HAM ? 0 : (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
   int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
-  uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + 32);             // 32 keys
+  uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + (MS ? 32 * MAX_STEPS : 32));  // 32 keys
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
   uint64_t* qa = ev + 32;                                               // QR == 0 only
   uint64_t* qb = qa + (QR == 0 ? L : 0);
@@ -962,15 +965,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
             in_topk |= __any_sync(FULL, b0 + lane < tsize && tk[b0 + lane] == now);
         }
       }
-      if (QR > 0) {
-        if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
-        q.pop_front(lane);
-      } else if (!in_topk) {
-        evicted = (tsize == L) ? tk[L - 1] : KEY_MAX;
+      // push x into the shared-memory topk (L > 128); returns the evicted key
+      auto smem_topk_push = [&](uint64_t x) -> uint64_t {
+        const uint64_t out = (tsize == L) ? tk[L - 1] : KEY_MAX;
         int pos = 0;
         for (int b0 = 0; b0 < tsize; b0 += 32) {
           int i = b0 + lane;
-          pos += __popc(__ballot_sync(FULL, i < tsize && tk[i] < now));
+          pos += __popc(__ballot_sync(FULL, i < tsize && tk[i] < x));
         }
         const int newsize = min(tsize + 1, L);
         for (int b0 = ((newsize - 1) >> 5) << 5; b0 >= ((pos >> 5) << 5); b0 -= 32) {
@@ -981,18 +982,47 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
             val = tk[i - 1];
             w = true;
           } else if (i == pos) {
-            val = now;
+            val = x;
             w = true;
           }
           __syncwarp();
           if (w) tk[i] = val;
         }
+        return out;
+      };
+      if (QR > 0) {
+        if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
+        q.pop_front(lane);
+      } else if (!in_topk) {
+        evicted = smem_topk_push(now);
       }
       if (!in_topk) tsize = min(tsize + 1, L);
       if (DEL) v_erase_lane0(evicted);  // §IV-E: topk's evicted vertex
       __syncwarp();
-      const int na = qsize - 1;  // q after the pop
-      const uint64_t* A = qa + 1;
+      // multi-step probing (§V, R13): up to a.steps pops, each checked
+      // against the termination rule with topk as the previous pops left it
+      int npop = 1;
+      int popid = key_id(now);  // lane i < npop: id of the i-th popped vertex
+      if constexpr (MS) {
+        for (; npop < a.steps && npop < qsize; ++npop) {
+          const uint64_t nx = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : qa[npop];
+          const uint64_t tm = (QR > 0) ? tk_r.get(L - 1) : ((tsize == L) ? tk[L - 1] : KEY_MAX);
+          if (tm < nx) break;
+          uint64_t ev1;
+          if (QR > 0) {
+            ev1 = tk_r.insert_one(nx, L, lane);
+            q.pop_front(lane);
+          } else {
+            ev1 = smem_topk_push(nx);
+          }
+          tsize = min(tsize + 1, L);
+          if (DEL) v_erase_lane0(ev1);
+          __syncwarp();
+          if (lane == npop) popid = key_id(nx);
+        }
+      }
+      const int na = qsize - npop;  // q after the pops
+      const uint64_t* A = qa + npop;
 
       // ---- a4: candidate locating (§V)
       int v = adjv;
@@ -1005,18 +1035,50 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
       const bool seen = v_contains(v, keep);
       keep = keep && !seen;
       const unsigned km = __ballot_sync(FULL, keep);
-      const int nc = __popc(km);
+      int nc_all = __popc(km);
       if (keep) cid[__popc(km & lt)] = v;
       __syncwarp();
+      if constexpr (MS) {
+        // the other popped rows, in pop order: one candidate list (R13)
+        for (int i = 1; i < npop; ++i) {
+          const int pid = __shfl_sync(FULL, popid, i);
+          int v2 = (lane < a.degree) ? __ldg(a.adj + (int64_t)pid * a.degree + lane) : -1;
+          bool k2 = v2 >= 0;
+          if (a.dedup) {
+            const unsigned grp = __match_any_sync(FULL, v2);
+            k2 = k2 && ((grp & lt) == 0);
+          }
+          bool dup = false;  // already located from an earlier popped row
+          for (int j = 0; j < nc_all; ++j) dup |= (cid[j] == v2);
+          k2 = k2 && !dup;
+          const bool seen2 = v_contains(v2, k2);
+          k2 = k2 && !seen2;
+          const unsigned m2 = __ballot_sync(FULL, k2);
+          if (k2) cid[nc_all + __popc(m2 & lt)] = v2;
+          nc_all += __popc(m2);
+          __syncwarp();
+        }
+      }
+      n_dist += nc_all;
+      n_exp += npop;
+      // distance + maintenance over groups of <= 32 candidates (one group
+      // unless multi-step probing located more): for the exact hash and the
+      // insert-only Bloom filter the result of a batch does not depend on
+      // how it is split (the selection threshold is fixed within an iteration
+      // and evictions = (q u new) minus its L smallest)
+      int na_g = na;
+      const uint64_t* A_g = A;
+      for (int g0 = 0;; g0 += 32) {
+      const int nc = min(32, nc_all - g0);
+      const int* cidg = cid + g0;
+      const bool last_group = !MS || g0 + 32 >= nc_all;
 
       // ---- a5: bulk distance computation (§VI)
       const float dist =
-          bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, nc, qv, stage, a.cosine, lane);
-      n_dist += nc;
-      n_exp += 1;
+          bulk_distance<NCH, METRIC>(a.data, a.dpad, cidg, nc, qv, stage, a.cosine, lane);
 
       // ---- a6: maintenance (§IV-C/D/E)
-      const int myid = lane < nc ? cid[lane] : -1;
+      const int myid = lane < nc ? cidg[lane] : -1;
       uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
       const uint64_t thr =
           (a.sel && tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
@@ -1027,8 +1089,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
       const int ns = __popc(smask);
       if (!sel) key = KEY_MAX;
       // prefetch the adjacency row of the next head = min(q head, best new key)
-      {
-        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na > 0 ? A[0] : KEY_MAX);
+      if (last_group) {
+        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na_g > 0 ? A_g[0] : KEY_MAX);
         uint64_t nxt = umin64(qhead, warp_min_key(key));
         if (nxt != KEY_MAX && lane < a.degree)
           adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
@@ -1063,19 +1125,19 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
                 hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
               }
             } else {
-              for (int i0 = 0; i0 < na; i0 += 32)
-                hs.insert(i0 + lane < na ? key_id(A[i0 + lane]) : 0, i0 + lane < na);
+              for (int i0 = 0; i0 < na_g; i0 += 32)
+                hs.insert(i0 + lane < na_g ? key_id(A_g[i0 + lane]) : 0, i0 + lane < na_g);
               for (int i0 = 0; i0 < tsize; i0 += 32)
                 hs.insert(i0 + lane < tsize ? key_id(tk[i0 + lane]) : 0, i0 + lane < tsize);
             }
-            used = na + tsize;
+            used = na_g + tsize;
             __syncwarp();
           }
           const bool took = hs.insert(myid, sel);
           used += __popc(__ballot_sync(FULL, took));
         }
       };
-      int qsize_new = min(na + ns, L);
+      int qsize_new = min(na_g + ns, L);
       if (QR > 0) {
         if (ns > 0) {  // (ns == 0: q only lost its head, nothing to insert/evict)
           visit_selected();
@@ -1092,7 +1154,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
             }
           }
           const int nq_new = __popc(qmask);
-          qsize_new = min(na + nq_new, L);
+          qsize_new = min(na_g + nq_new, L);
           // compact the selected keys to lanes [0, nq_new), sort only those
           if ((qmask >> lane) & 1u) keys32[__popc(qmask & lt)] = key;
           __syncwarp();
@@ -1137,8 +1199,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         int nsq = ns;  // selected keys that enter q
         if constexpr (VK == VK_CUCKOO) {
           // drop keys already in q (Cuckoo false negatives), re-compact
-          const int j = count_below(A, na, key);
-          const bool dup = lane < ns && j < na && A[j] == key;
+          const int j = count_below(A_g, na_g, key);
+          const bool dup = lane < ns && j < na_g && A_g[j] == key;
           const unsigned keepm = __ballot_sync(FULL, lane < ns && !dup);
           nsq = __popc(keepm);
           __syncwarp();
@@ -1150,29 +1212,33 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         keys32[lane] = key;
         __syncwarp();
         // merged position p >= L is evicted: ev[p - L] (< 32 of them) in key order
-        for (int i0 = 0; i0 < na; i0 += 32) {
+        for (int i0 = 0; i0 < na_g; i0 += 32) {
           const int i = i0 + lane;
-          const uint64_t x = i < na ? A[i] : KEY_MAX;
+          const uint64_t x = i < na_g ? A_g[i] : KEY_MAX;
           const int p = i + count_below(keys32, nsq, x);
-          if (i < na && p < L) qb[p] = x;
-          if (i < na && p >= L) ev[p - L] = x;
-          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na && p >= L);
+          if (i < na_g && p < L) qb[p] = x;
+          if (i < na_g && p >= L) ev[p - L] = x;
+          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na_g && p >= L);
         }
         {
-          const int p = lane + count_below(A, na, key);
+          const int p = lane + count_below(A_g, na_g, key);
           if (lane < nsq && p < L) qb[p] = key;
           if (lane < nsq && p >= L) ev[p - L] = key;
           if constexpr (VK == VK_HASH) hs.erase(key_id(key), lane < nsq && p >= L);
         }
         __syncwarp();
-        if constexpr (VK == VK_CUCKOO) cuckoo_erase_sorted_desc(max(0, na + nsq - L));
-        qsize_new = min(na + nsq, L);
+        if constexpr (VK == VK_CUCKOO) cuckoo_erase_sorted_desc(max(0, na_g + nsq - L));
+        qsize_new = min(na_g + nsq, L);
         uint64_t* t = qa;
         qa = qb;
         qb = t;
       }
       qsize = qsize_new;
       __syncwarp();
+      na_g = qsize;
+      A_g = qa;
+      if (last_group) break;
+      }  // candidate groups
       if (VK == VK_GHASH && used > (1 << (a.table_log2 - 1))) {  // keep load <= 1/2
         full = true;
         break;

@@ -170,6 +170,7 @@ struct Shape {
 };
 
 Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
+  const int steps = p->steps;
   Shape s;
   int tbytes = 0;
   s.rebuild_at = 0;
@@ -201,8 +202,9 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
-  s.warp_bytes = stage_bytes + 16 + 32 * 4 + 32 * 8 + 32 * 8 + (s.qr == 0 ? 3 * L * 8 + 8 : 0) +
-                 tbytes;
+  const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
+  s.warp_bytes = stage_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
+                 (s.qr == 0 ? 3 * L * 8 + 8 : 0) + tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;
 }
@@ -223,6 +225,12 @@ int check_params(const song_index* ix, const song_search_params* p) {
   if (p->warps_per_block < 0 || p->warps_per_block > SONG_LB_THREADS / 32)
     return fail(SONG_EINVAL, "warps_per_block %d outside [0, %d]", p->warps_per_block, SONG_LB_THREADS / 32);
   if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
+  if (p->steps < 0) return fail(SONG_EINVAL, "steps %d < 0", p->steps);
+  if (p->steps > SONG_MAX_STEPS)
+    return fail(SONG_EUNSUPPORTED, "steps %d > %d", p->steps, SONG_MAX_STEPS);
+  if (p->steps > 1 && ((p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM) ||
+                       ix->metric == SONG_HAMMING))
+    return fail(SONG_EUNSUPPORTED, "multi-step probing needs visited HASH or BLOOM on a float index");
   return SONG_OK;
 }
 
@@ -266,6 +274,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.entry = p->entry;
   a.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);
   a.id_offset = p->id_offset;
+  a.steps = p->steps > 1 ? p->steps : 1;
   int warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
   while (warps > 1 && (size_t)sh.warp_bytes * warps > 200 * 1024) warps >>= 1;
   if ((size_t)sh.warp_bytes * warps > 227 * 1024)

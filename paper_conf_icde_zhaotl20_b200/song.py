@@ -47,7 +47,8 @@ class SearchParams(ctypes.Structure):
                 ("visited", ctypes.c_int32), ("bloom_log2_bits", ctypes.c_int32),
                 ("entry", ctypes.c_int32), ("max_iters", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
-                ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32)]
+                ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32),
+                ("steps", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -135,6 +136,7 @@ class Params:
     blocks_per_sm: int = 0
     id_offset: int = 0
     table_log2: int = 0
+    steps: int = 1  # multi-step probing (pops per iteration, §V)
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -147,6 +149,7 @@ class Params:
         p.blocks_per_sm = self.blocks_per_sm
         p.id_offset = self.id_offset
         p.table_log2 = self.table_log2
+        p.steps = self.steps
         return p
 
 

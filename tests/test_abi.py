@@ -52,7 +52,7 @@ def test_argument_errors_need_no_gpu():
     assert lib.song_index_destroy(None) == 0
     p = song.SearchParams()
     lib.song_default_params(ctypes.byref(p), 10, 64)
-    assert (p.K, p.queue_len, p.visited, p.entry, p.id_offset) == (10, 64, 0, 0, 0)
+    assert (p.K, p.queue_len, p.visited, p.entry, p.id_offset, p.steps) == (10, 64, 0, 0, 0, 0)
 
 
 def test_params_struct_layout_matches_header(tmp_path):
