@@ -6,7 +6,7 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R13 it follows are listed in its header and in DESIGN.md §3).
+R1-R14 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
@@ -35,11 +35,13 @@ SEL = 2
 DEL = 4
 BLOOM = 8
 CUCKOO = 16
+LAZY = 32   # with DEL: deletions deferred until visited reaches lazy_cap (reading R14)
 OPTIMIZED = BOUNDED_Q | SEL | DEL          # "hashtable-sel-del" (Fig. 7)
 OPTIMIZED_BLOOM = BOUNDED_Q | SEL | BLOOM  # "bloomfilter" (Fig. 7)
 OPTIMIZED_CUCKOO = BOUNDED_Q | SEL | DEL | CUCKOO  # "cuckoofilter" (Fig. 7)
 HASHTABLE = BOUNDED_Q                      # "hashtable" (Fig. 7): no sel, no del
 HASHTABLE_SEL = BOUNDED_Q | SEL            # "hashtable-sel" (Fig. 7)
+OPTIMIZED_LAZY = OPTIMIZED | LAZY          # hash-sel-del with lazy deletion (R14)
 
 _TRACE_FN = ctypes.CFUNCTYPE(
     None, ctypes.c_void_p, ctypes.c_int64,
@@ -74,8 +76,8 @@ def _load():
         lib.oracle_search_steps.argtypes = [
             P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, ctypes.c_int32,
             P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
-            ctypes.c_int64, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P,
-            ctypes.c_int32, _TRACE_FN, P]
+            ctypes.c_int64, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int64,
+            P, P, P, ctypes.c_int32, _TRACE_FN, P]
         lib.oracle_distance.restype = ctypes.c_float
         lib.oracle_distance.argtypes = [P, P, ctypes.c_int32, ctypes.c_int32]
         lib.oracle_bruteforce.restype = None
@@ -131,11 +133,13 @@ def default_bloom_bits(L: int) -> int:
 
 def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OPTIMIZED,
            bloom_bits: Optional[int] = None, entry: int = 0, max_iters: int = 1 << 40,
-           nthreads: int = 1, trace: Optional[Callable] = None, steps: int = 1):
+           nthreads: int = 1, trace: Optional[Callable] = None, steps: int = 1,
+           lazy_cap: int = 0):
     """Run the oracle.  Returns (ids [nq,K] int32, dists [nq,K] f32,
     counters [nq,2] int64 = (n_dist, n_exp), n_capped).  ``bloom_bits`` is the
     Bloom filter's bit count, or the Cuckoo filter's bucket count; ``steps`` is
-    the multi-step probing width (pops per iteration, reading R13)."""
+    the multi-step probing width (pops per iteration, reading R13); ``lazy_cap``
+    the visited capacity of the LAZY flag (reading R14)."""
     lib = _load()
     data = _f32(data)
     adj = _i32(adj)
@@ -162,7 +166,8 @@ def search(data, adj, queries, K: int, L: int, metric: int = L2, flags: int = OP
         cb = _TRACE_FN(_cb)
     capped = lib.oracle_search_steps(_ptr(data), n, dim, _ptr(adj), degree, metric,
                                      _ptr(queries), nq, K, L, flags, int(bloom_bits), entry,
-                                     int(max_iters), int(steps), _ptr(ids), _ptr(dists),
+                                     int(max_iters), int(steps), int(lazy_cap), _ptr(ids),
+                                     _ptr(dists),
                                      _ptr(counters), int(nthreads), cb, None)
     return ids, dists, counters, int(capped)
 

@@ -43,6 +43,14 @@
 //      previous pops), locates the unvisited neighbours of all of them into ONE
 //      candidate list (pop order, then row order, first occurrence), then runs
 //      the distance and maintenance stages once.  n_exp counts pops.
+//   R14 lazy visited deletion (a B200 schedule of P:435, flag ORACLE_LAZY with
+//      DEL): the erasures of §IV-E are deferred; when inserting an iteration's
+//      selected candidates would grow the exact visited set past a capacity C,
+//      visited := ids(q) ∪ ids(topk) first (every deferred erasure at once).
+//      Any schedule of the erasures leaves the result unchanged (a vertex
+//      evicted from q ∪ topk has L better vertices there for good), so only
+//      the counters move: fewer recomputed distances than eager deletion,
+//      memory still bounded by C >= 2L + 32.
 //   R12 Hamming search: the distance of two codes is the number of differing
 //      bits ("the hamming distance between the bit-vectors"), used as the
 //      key's distance (an integer, exact in fp32) with the same (dist, id)
@@ -75,6 +83,7 @@ enum Flags {
   ORACLE_DEL = 4,        // §IV-E: visited deletion
   ORACLE_BLOOM = 8,      // §IV-B: visited is a Bloom filter (no deletion)
   ORACLE_CUCKOO = 16,    // visited is a Cuckoo filter (supports deletion)
+  ORACLE_LAZY = 32,      // with DEL: deletions deferred until visited reaches a capacity (R14)
 };
 
 struct Key {
@@ -286,6 +295,7 @@ struct Problem {
   uint64_t bloom_bits;  // Bloom: bits; Cuckoo: buckets
   int64_t max_iters;
   int steps;            // multi-step probing: pops per iteration (R13), >= 1
+  int64_t lazy_cap;     // ORACLE_LAZY: visited capacity (R14)
 };
 
 // Algorithm 1 with the optimizations of §IV switched by flags.
@@ -296,7 +306,8 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
   const int L = P.L;
   const bool bounded = P.flags & ORACLE_BOUNDED_Q;
   const bool sel = P.flags & ORACLE_SEL;
-  const bool del = P.flags & ORACLE_DEL;
+  const bool lazy = (P.flags & ORACLE_LAZY) && (P.flags & ORACLE_DEL);
+  const bool del = (P.flags & ORACLE_DEL) && !lazy;  // eager deletion
   Visited visited((P.flags & ORACLE_BLOOM) ? 1 : (P.flags & ORACLE_CUCKOO) ? 2 : 0, P.bloom_bits,
                   P.bloom_bits);
   std::set<Key> q;     // min-priority queue (begin() = min, prev(end()) = max)
@@ -367,9 +378,24 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
     // structure maintenance stage uses the distances to update the priority
     // queues and the hash table"): insert the selected candidates in
     // candidate order, then evict q's maximum while |q| > L.
-    for (const Key& k : ck) {
+    auto selected = [&](const Key& k) {
       // [sel] P:429: filtered when topk is full and k is worse than all of it (R3).
-      if (sel && (int)topk.size() == L && *std::prev(topk.end()) < k) continue;
+      return !(sel && (int)topk.size() == L && *std::prev(topk.end()) < k);
+    };
+    if (lazy) {
+      // R14: the deferred deletions of P:435 are applied all at once — visited
+      // becomes ids(q) ∪ ids(topk), the set eager deletion would hold — when
+      // inserting this iteration's selected candidates would pass the capacity
+      int64_t n_sel = 0;
+      for (const Key& k : ck) n_sel += selected(k);
+      if (n_sel > 0 && (int64_t)visited.exact.size() + n_sel > P.lazy_cap) {
+        visited.exact.clear();
+        for (const Key& k : q) visited.exact.insert(k.id);
+        for (const Key& k : topk) visited.exact.insert(k.id);
+      }
+    }
+    for (const Key& k : ck) {
+      if (!selected(k)) continue;
       visited.insert(k.id);
       q.insert(k);
     }
@@ -409,11 +435,12 @@ extern "C" {
 int64_t oracle_search_steps(const float* data, int64_t n, int32_t dim, const int32_t* adj,
                             int32_t degree, int32_t metric, const float* queries, int64_t nq,
                             int32_t K, int32_t L, int32_t flags, int64_t bloom_bits,
-                            int32_t entry, int64_t max_iters, int32_t steps, int32_t* ids,
+                            int32_t entry, int64_t max_iters, int32_t steps, int64_t lazy_cap,
+                            int32_t* ids,
                             float* dists, int64_t* counters, int32_t nthreads, trace_fn cb,
                             void* ctx) {
   Problem P{data, n, dim, adj, degree, metric, K, L, flags, entry, (uint64_t)bloom_bits, max_iters,
-            steps < 1 ? 1 : steps};
+            steps < 1 ? 1 : steps, lazy_cap};
   if (nthreads <= 1 || cb) {
     int64_t fails = 0;
     for (int64_t i = 0; i < nq; ++i)
@@ -447,8 +474,8 @@ int64_t oracle_search(const float* data, int64_t n, int32_t dim, const int32_t* 
                       int64_t max_iters, int32_t* ids, float* dists, int64_t* counters,
                       int32_t nthreads, trace_fn cb, void* ctx) {
   return oracle_search_steps(data, n, dim, adj, degree, metric, queries, nq, K, L, flags,
-                             bloom_bits, entry, max_iters, 1, ids, dists, counters, nthreads, cb,
-                             ctx);
+                             bloom_bits, entry, max_iters, 1, 0, ids, dists, counters, nthreads,
+                             cb, ctx);
 }
 
 // The distance of §VI for one pair (exposed so tests can pin R7 directly).
