@@ -103,6 +103,18 @@ typedef struct song_search_params {
                               list; 0 or 1 = Algorithm 1's single pop; at most
                               SONG_MAX_STEPS; > 1 needs visited HASH or BLOOM and a
                               float index (else SONG_EUNSUPPORTED) */
+  int32_t visited_cap;     /* SONG_VISITED_HASH deletion schedule (§IV-E, DESIGN.md
+                              reading R14).  0 = lazy deletion with the default capacity
+                              C = S/2 for queue_len <= 128, 3S/4 above, where S =
+                              2^ceil(log2(F (2L + 32))) table slots, F = 8 (L <= 128) or
+                              2; > 0 = lazy with C = visited_cap (2L + 32 <= C <= 3S/4,
+                              else SONG_EINVAL); -1 = eager deletion (every evicted vertex
+                              erased at once, the paper's literal schedule).  Lazy: the
+                              erasures are applied together (visited := ids(q) ∪
+                              ids(topk)) when the selected candidates of an iteration
+                              would grow visited past C — same results, fewer recomputed
+                              distances.  steps > 1 always uses eager deletion.  Ignored
+                              by the other visited kinds. */
 } song_search_params;
 
 typedef struct song_index_info {

@@ -64,6 +64,7 @@ struct SearchArgs {
   int table_log2;  // hash: log2 slots; bloom: log2 bits
   int entry, max_iters, id_offset;
   int steps;       // multi-step probing (§V, reading R13): pops per iteration
+  int lazy;        // VK_HASH: deletions deferred to the rebuild at rebuild_at (reading R14)
   int cosine;      // MET_DOT: 1 -> 1 - dot, 0 -> -dot
   int dedup;       // 1 if some adjacency row repeats an id
   int rebuild_at;  // hash: rebuild when live + tombstones would exceed this
@@ -833,7 +834,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
     }
   };
   auto v_erase_lane0 = [&](uint64_t k) {
-    if constexpr (VK == VK_HASH) hs.erase(key_id(k), k != KEY_MAX && lane == 0);
+    if constexpr (VK == VK_HASH) hs.erase(key_id(k), k != KEY_MAX && lane == 0 && !a.lazy);
     if constexpr (VK == VK_CUCKOO) {
       if (lane == 0 && k != KEY_MAX) cs.erase1(key_id(k));
       __syncwarp();
@@ -1115,7 +1116,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         }
         if constexpr (VK == VK_HASH) {
           if (used + ns > a.rebuild_at) {
-            // tombstones accumulated: rebuild visited = ids(q) ∪ ids(topk)
+            // tombstones accumulated (eager deletion) or the capacity is reached
+            // (lazy deletion, R14): rebuild visited = ids(q) ∪ ids(topk)
             for (int i = lane; i < twords; i += 32) table[i] = EMPTY;
             __syncwarp();
             if (QR > 0) {
@@ -1168,7 +1170,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
 #pragma unroll
           for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
             const bool beyond = r * 32 + lane >= L && q.v[r] != KEY_MAX;
-            if constexpr (VK == VK_HASH) hs.erase(key_id(q.v[r]), beyond);
+            if constexpr (VK == VK_HASH) hs.erase(key_id(q.v[r]), beyond && !a.lazy);
             if constexpr (VK == VK_CUCKOO) {
               const unsigned bm = __ballot_sync(FULL, beyond);
               if (beyond) ev[ne + __popc(bm & lt)] = q.v[r];
@@ -1176,7 +1178,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
             }
             q.v[r] = r * 32 + lane >= L ? KEY_MAX : q.v[r];
           }
-          if constexpr (VK == VK_HASH) hs.erase(key_id(out), out != KEY_MAX);
+          if constexpr (VK == VK_HASH) hs.erase(key_id(out), out != KEY_MAX && !a.lazy);
           if constexpr (VK == VK_CUCKOO) {
             const bool o = out != KEY_MAX;
             const unsigned bm = __ballot_sync(FULL, o);
@@ -1218,13 +1220,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
           const int p = i + count_below(keys32, nsq, x);
           if (i < na_g && p < L) qb[p] = x;
           if (i < na_g && p >= L) ev[p - L] = x;
-          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na_g && p >= L);
+          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na_g && p >= L && !a.lazy);
         }
         {
           const int p = lane + count_below(A_g, na_g, key);
           if (lane < nsq && p < L) qb[p] = key;
           if (lane < nsq && p >= L) ev[p - L] = key;
-          if constexpr (VK == VK_HASH) hs.erase(key_id(key), lane < nsq && p >= L);
+          if constexpr (VK == VK_HASH) hs.erase(key_id(key), lane < nsq && p >= L && !a.lazy);
         }
         __syncwarp();
         if constexpr (VK == VK_CUCKOO) cuckoo_erase_sorted_desc(max(0, na_g + nsq - L));

@@ -162,6 +162,7 @@ int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* a
 #endif
 // per-warp shared memory of the search kernel
 struct Shape {
+  int lazy = 0;
   int table_log2;
   int rebuild_at;
   int warp_bytes;
@@ -193,6 +194,11 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     const bool big = L > 128;
     s.table_log2 = next_pow2_log2((big ? 2ll : (long long)SONG_HASH_FACTOR) * (2 * L + 32));
     s.rebuild_at = big ? (3 << s.table_log2) / 4 : (SONG_HASH_REBUILD_NUM << s.table_log2) / 16;
+    // lazy deletion (R14): visited holds up to C live ids, no tombstones
+    s.lazy = p->visited_cap >= 0 && p->steps <= 1;
+    if (s.lazy)
+      s.rebuild_at = p->visited_cap > 0 ? p->visited_cap
+                                        : (big ? (3 << s.table_log2) / 4 : (1 << s.table_log2) / 2);
     tbytes = (1 << s.table_log2) * 4;
   }
   // float rows: NCH = 16 B chunks per lane (128 floats per chunk row);
@@ -226,6 +232,15 @@ int check_params(const song_index* ix, const song_search_params* p) {
     return fail(SONG_EINVAL, "warps_per_block %d outside [0, %d]", p->warps_per_block, SONG_LB_THREADS / 32);
   if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
   if (p->steps < 0) return fail(SONG_EINVAL, "steps %d < 0", p->steps);
+  if (p->visited_cap < -1) return fail(SONG_EINVAL, "visited_cap %d < -1", p->visited_cap);
+  if (p->visited_cap > 0 && p->visited == SONG_VISITED_HASH) {
+    const bool big = p->queue_len > 128;
+    const int slots = 1 << next_pow2_log2((big ? 2ll : (long long)SONG_HASH_FACTOR) *
+                                          (2ll * p->queue_len + 32));
+    if (p->visited_cap < 2 * p->queue_len + 32 || p->visited_cap > 3 * (slots / 4))
+      return fail(SONG_EINVAL, "visited_cap %d outside [2L + 32, 3/4 of %d slots]",
+                  p->visited_cap, slots);
+  }
   if (p->steps > SONG_MAX_STEPS)
     return fail(SONG_EUNSUPPORTED, "steps %d > %d", p->steps, SONG_MAX_STEPS);
   if (p->steps > 1 && ((p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM) ||
@@ -270,6 +285,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   Shape sh = search_shape(p->queue_len, vk, p, ix->dpad, ix->metric == SONG_HAMMING);
   a.table_log2 = sh.table_log2;
   a.rebuild_at = sh.rebuild_at;
+  a.lazy = sh.lazy;
   a.warp_smem_bytes = sh.warp_bytes;
   a.entry = p->entry;
   a.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);

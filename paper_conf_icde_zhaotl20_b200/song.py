@@ -48,7 +48,7 @@ class SearchParams(ctypes.Structure):
                 ("entry", ctypes.c_int32), ("max_iters", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32),
-                ("steps", ctypes.c_int32)]
+                ("steps", ctypes.c_int32), ("visited_cap", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -137,6 +137,7 @@ class Params:
     id_offset: int = 0
     table_log2: int = 0
     steps: int = 1  # multi-step probing (pops per iteration, §V)
+    visited_cap: int = 0  # hash deletion schedule: 0 lazy (default cap), >0 lazy cap, -1 eager
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -150,6 +151,7 @@ class Params:
         p.id_offset = self.id_offset
         p.table_log2 = self.table_log2
         p.steps = self.steps
+        p.visited_cap = self.visited_cap
         return p
 
 
@@ -312,6 +314,16 @@ def merge_topk(ids, dists, K: int):
                                  G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
                                  ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
     return oi, od
+
+
+def default_visited_cap(L: int) -> int:
+    """The default lazy-deletion capacity C of include/song.h (visited_cap = 0)."""
+    big = L > 128
+    need = (2 if big else 8) * (2 * L + 32)
+    slots = 1
+    while slots < need:
+        slots <<= 1
+    return 3 * slots // 4 if big else slots // 2
 
 
 def rp_encode(vectors, R):

@@ -32,6 +32,26 @@ ORACLE_FLAGS = {"hash": oracle.OPTIMIZED, "bloom": oracle.OPTIMIZED_BLOOM,
 ALL_VISITED = list(ORACLE_FLAGS)
 
 
+def lazy_cap_for(L):
+    """include/song.h's default lazy-deletion capacity (visited_cap = 0):
+    S/2 for L <= 128, 3S/4 above, S = 2^ceil(log2(F (2L + 32))), F = 8 or 2."""
+    big = L > 128
+    slots = 1 << int(np.ceil(np.log2((2 if big else 8) * (2 * L + 32))))
+    return 3 * slots // 4 if big else slots // 2
+
+
+def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0):
+    """The oracle mode matching a GPU search: the hash's deletion schedule is
+    lazy (reading R14) unless visited_cap = -1 or steps > 1 (eager)."""
+    kw = dict(flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L, log2, visited))
+    if visited == "hash" and steps <= 1 and visited_cap >= 0:
+        kw["flags"] = oracle.OPTIMIZED_LAZY
+        kw["lazy_cap"] = visited_cap or lazy_cap_for(L)
+    if steps > 1:
+        kw["steps"] = steps
+    return kw
+
+
 def gpu_search(idx, q, K, L, visited="hash", allow_cap=False, **kw):
     s = song()
     p = s.Params(K=K, queue_len=L, visited=visited, **kw)
@@ -83,7 +103,7 @@ def test_fig1_toy_on_gpu(visited):
     if visited == "hash":
         assert c[0].tolist() == [12, 4]  # Fig. 4(c): 12 distances, 4 expansions
     o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
-                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(3, visited=visited))
+                      **oracle_kw(visited, 3))
     assert_exact((ids, d, c), o)
 
 
@@ -105,8 +125,7 @@ def test_tiny_parity(tiny, L, visited):
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q, cfg.K, L, visited)
-    o = oracle.search(x, adj, q, cfg.K, L, flags=ORACLE_FLAGS[visited],
-                      bloom_bits=bloom_bits_for(L, visited=visited))
+    o = oracle.search(x, adj, q, cfg.K, L, **oracle_kw(visited, L))
     assert_close(g, o, truth, scale=float(np.abs(o[1]).max()))
 
 
@@ -130,7 +149,7 @@ def test_sift_integer_bit_exact(sift100k, L, visited, warps):
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q.cpu().numpy(), cfg.K, L, visited, warps_per_block=warps)
     o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, L,
-                      flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L, visited=visited),
+                      **oracle_kw(visited, L),
                       nthreads=8)
     assert_exact(g, o)
 
@@ -226,8 +245,7 @@ def test_edges_exact(dim, L, K):
     idx = s.SongIndex(x, adj)
     for visited in ALL_VISITED:
         g = gpu_search(idx, q, K, L, visited)
-        o = oracle.search(x, adj, q, K, L, flags=ORACLE_FLAGS[visited],
-                          bloom_bits=bloom_bits_for(L, visited=visited))
+        o = oracle.search(x, adj, q, K, L, **oracle_kw(visited, L))
         assert_exact(g, o)
 
 
@@ -250,6 +268,9 @@ def test_large_queue_len_max():
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q[:16], 100, 2048)
+    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048))
+    assert_exact(g, o)
+    g = gpu_search(idx, q[:16], 100, 2048, visited_cap=-1)  # eager deletion
     o = oracle.search(x, adj, q[:16], 100, 2048)
     assert_exact(g, o)
 
@@ -327,6 +348,26 @@ def test_dataset_sharding_emulated_on_one_gpu(sift100k):
     np.testing.assert_array_equal(md.cpu().numpy(), ed)
 
 
+@pytest.mark.parametrize("L", [10, 48, 64, 128, 200])
+@pytest.mark.parametrize("cap", [-1, 0, "min"])
+def test_deletion_schedules_exact(sift100k, L, cap):
+    """Reading R14: eager (-1), default lazy (0) and the smallest lazy capacity
+    2L + 32 — identical results, each schedule's own counters bit-exact."""
+    cfg, x, q, adj = sift100k
+    cap = 2 * L + 32 if cap == "min" else cap
+    s = song()
+    idx = s.SongIndex(x, adj)
+    xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()
+    g = gpu_search(idx, qn, cfg.K, L, "hash", visited_cap=cap)
+    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap))
+    assert_exact(g, o)
+    eager = oracle.search(xn, an, qn, cfg.K, L, nthreads=8)
+    np.testing.assert_array_equal(g[0], eager[0])  # the schedule never changes results
+    np.testing.assert_array_equal(g[1], eager[1])
+    if cap != -1:
+        assert g[2][:, 0].sum() <= eager[2][:, 0].sum()  # ... only the recomputations
+
+
 @pytest.mark.slow
 def test_sift1m_full_size_sampled_parity():
     """BASELINE configs[1] at full size (1M x 128, degree 32, 10,000 queries) in
@@ -344,7 +385,8 @@ def test_sift1m_full_size_sampled_parity():
     rng = np.random.default_rng(0)
     pick = np.sort(rng.choice(cfg.nq, 300, replace=False))
     xn, an = x.cpu().numpy(), adj.cpu().numpy()
-    o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 48, nthreads=8)
+    o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 48, nthreads=8,
+                      **oracle_kw("hash", 48))
     assert_exact((ids.cpu().numpy()[pick], d.cpu().numpy()[pick], c.cpu().numpy()[pick]), o)
     # properties that hold for every query at any size: sorted, unique, valid ids
     ii, dd = ids.cpu().numpy(), d.cpu().numpy()

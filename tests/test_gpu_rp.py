@@ -79,8 +79,8 @@ def test_hamming_search_bit_exact(mnist, bits, L, visited):
                                  s.Params(K=K, queue_len=L, visited=visited), counters=True)
     torch.cuda.synchronize()
     idx.last_status()
-    flags = oracle.OPTIMIZED if visited == "hash" else oracle.OPTIMIZED_BLOOM
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, K, L, flags=flags, nthreads=8)
+    from test_gpu_parity import oracle_kw
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, K, L, nthreads=8, **oracle_kw(visited, L))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
@@ -108,7 +108,8 @@ def test_rp_index_end_to_end(mnist, monkeypatch, chunk_rows):
     idx.last_status()
     codes = oracle.rp_encode(x, R, nthreads=8)
     qc = oracle.rp_encode(q, R, nthreads=8)
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 1, 64, nthreads=8)
+    from test_gpu_parity import oracle_kw
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 1, 64, nthreads=8, **oracle_kw("hash", 64))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
@@ -135,7 +136,7 @@ def test_hamming_errors(mnist):
                               s.Params(K=5, queue_len=16))
     torch.cuda.synchronize()
     assert (d.cpu().numpy() == 0).all()
-    oi, od, _, _ = oracle.search_codes(codes, adj, np.zeros((2, 4), np.uint32), 5, 16)
+    oi, od, _, _ = oracle.search_codes(codes, adj, np.zeros((2, 4), np.uint32), 5, 16)  # ids only
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     idx.close()
 
@@ -158,7 +159,8 @@ def test_code_footprint_is_table4s(mnist, bits):
     ids, d, c = idx.search_codes(torch.as_tensor(qc.view(np.int32), device="cuda"),
                                  s.Params(K=5, queue_len=40), counters=True)
     torch.cuda.synchronize()
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 5, 40)
+    from test_gpu_parity import oracle_kw
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 5, 40, **oracle_kw("hash", 40))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
