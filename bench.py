@@ -44,6 +44,9 @@ def parse():
     ap.add_argument("--visited", default="hash", choices=["hash", "bloom"])
     ap.add_argument("--warps-per-block", type=int, default=0)
     ap.add_argument("--blocks-per-sm", type=int, default=0)
+    ap.add_argument("--visited-cap", type=int, default=0,
+                    help="hash deletion schedule: 0 lazy (default capacity), >0 lazy capacity, "
+                         "-1 eager (reading R14)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sweep-only", action="store_true")
@@ -238,7 +241,8 @@ def run_song(args, ws, rank, local, log):
 
     def params(L):
         return song.Params(K=cfg.K, queue_len=L, visited=args.visited,
-                           warps_per_block=args.warps_per_block, blocks_per_sm=args.blocks_per_sm)
+                           warps_per_block=args.warps_per_block, blocks_per_sm=args.blocks_per_sm,
+                           visited_cap=args.visited_cap)
 
     # ---- operating point: smallest grid queue_len with recall@10 >= target
     sweep = []
@@ -335,6 +339,7 @@ def run_song(args, ws, rank, local, log):
                         f"graph, {nq} queries/GPU, K={K}, queue_len={L_op}",
             "n": cfg.n, "dim": d, "degree": deg, "nq_per_gpu": nq, "K": K, "queue_len": L_op,
             "recall_at_10": round(rec, 4), "recall_sweep": sweep, "visited": args.visited,
+            "visited_cap": args.visited_cap or "default (lazy deletion, reading R14)",
             "l2": "flushed between timed steps (512 MiB write)",
             "parallelism": f"query-sharded dp{ws} (graph replicated per GPU)",
         },
@@ -362,10 +367,15 @@ def run_song(args, ws, rank, local, log):
     return result
 
 
-def oracle_mode(L):
-    """The oracle mode of the GPU's default hash schedule: selected insertion +
-    lazy visited deletion (reading R14) with include/song.h's default capacity."""
+def oracle_mode(L, cap=0):
+    """The oracle mode of the GPU's hash schedule: selected insertion + lazy
+    visited deletion (reading R14) with include/song.h's default capacity (or
+    `cap`; -1 = eager deletion)."""
     import oracle
+    if cap == -1:
+        return dict(flags=oracle.OPTIMIZED)
+    if cap > 0:
+        return dict(flags=oracle.OPTIMIZED_LAZY, lazy_cap=cap)
     big = L > 128
     slots = 1
     while slots < (2 if big else 8) * (2 * L + 32):
@@ -379,7 +389,7 @@ def cpu_baseline(args, x, adj, q, cfg, L, ids_c, dists_c, ctr, log):
     cores = len(os.sched_getaffinity(0))
     xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()
     t = time.perf_counter()
-    mode = oracle_mode(L)
+    mode = oracle_mode(L, args.visited_cap)
     oracle.search(xn, an, qn[:64], cfg.K, L, metric=oracle.METRICS[cfg.metric],
                   nthreads=cores, **mode)
     per_q = (time.perf_counter() - t) / 64

@@ -100,11 +100,16 @@ def test_fig1_toy_on_gpu(visited):
     idx = s.SongIndex(data, adj)
     ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited)
     assert [int(x) + 1 for x in ids[0]] == result
-    if visited == "hash":
-        assert c[0].tolist() == [12, 4]  # Fig. 4(c): 12 distances, 4 expansions
     o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
                       **oracle_kw(visited, 3))
     assert_exact((ids, d, c), o)
+    if visited == "hash":
+        # the paper's literal (eager) deletion: Fig. 4(c), 12 distances, 4 expansions
+        ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited, visited_cap=-1)
+        assert [int(x) + 1 for x in ids[0]] == result
+        assert c[0].tolist() == [12, 4]
+        # lazy deletion with the default capacity (R14): no vertex recomputed here
+        assert gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3)[2][0].tolist() == [10, 4]
 
 
 # ----------------------------------------------------------------- tiny config
