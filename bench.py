@@ -380,7 +380,7 @@ def oracle_mode(L, cap=0):
     slots = 1
     while slots < (2 if big else 8) * (2 * L + 32):
         slots <<= 1
-    return dict(flags=oracle.OPTIMIZED_LAZY, lazy_cap=3 * slots // 4 if big else slots // 2)
+    return dict(flags=oracle.OPTIMIZED_LAZY, lazy_cap=3 * slots // 4 if big else 5 * slots // 8)
 
 
 def cpu_baseline(args, x, adj, q, cfg, L, ids_c, dists_c, ctr, log):

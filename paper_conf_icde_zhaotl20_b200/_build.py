@@ -25,39 +25,50 @@ NVCC_FLAGS = [
 ]
 
 
-def _compile(src):
-    obj = os.path.join(BUILD, src.replace(".cu", ".o"))
-    cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-c",
-           "-o", obj, os.path.join(CSRC, src)]
+def _compile(src, defines=(), build_dir=BUILD):
+    obj = os.path.join(build_dir, src.replace(".cu", ".o"))
+    cmd = ["nvcc", *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"),
+           "-I", CSRC, "-c", "-o", obj, os.path.join(CSRC, src)]
     res = subprocess.run(cmd, capture_output=True, text=True)
     return src, obj, res
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB) -> str:
+    """Build libsong.so; ``defines``/``out`` build an experiment variant (A/B
+    measurements, e.g. SONG_DIST_V1) next to it without touching the default."""
     newest = max(os.path.getmtime(p) for p in DEPS)
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest:
-        return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    if not force and os.path.exists(out) and os.path.getmtime(out) >= newest:
+        return out
+    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.split("=")[0] for d in defines)
+    os.makedirs(build_dir, exist_ok=True)
     with concurrent.futures.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
-        results = list(ex.map(_compile, SOURCES))
+        results = list(ex.map(lambda src: _compile(src, defines, build_dir), SOURCES))
     report = []
     for src, obj, res in results:
         if res.returncode != 0:
             sys.stderr.write(res.stdout + res.stderr)
             raise RuntimeError(f"nvcc failed compiling {src}")
         report.append(res.stderr)
-    link = ["nvcc", "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", LIB,
+    link = ["nvcc", "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", out,
             *[obj for _, obj, _ in results]]
     res = subprocess.run(link, capture_output=True, text=True)
     if res.returncode != 0:
         sys.stderr.write(res.stdout + res.stderr)
         raise RuntimeError("nvcc failed linking libsong.so")
-    with open(os.path.join(PKG, "ptxas_report.txt"), "w") as f:
-        f.write("\n".join(report))
+    if out == LIB:
+        with open(os.path.join(PKG, "ptxas_report.txt"), "w") as f:
+            f.write("\n".join(report))
     if verbose:
         sys.stderr.write("\n".join(report))
-    return LIB
+    return out
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    import argparse
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--force", action="store_true")
+    ap.add_argument("-v", action="store_true")
+    ap.add_argument("--define", action="append", default=[])
+    ap.add_argument("--out", default=LIB)
+    a = ap.parse_args()
+    print(build(force=a.force, verbose=a.v, defines=a.define, out=a.out))

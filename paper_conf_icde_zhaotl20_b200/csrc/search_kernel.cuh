@@ -535,6 +535,11 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
 #ifndef SONG_STAGE_BUFS
 #define SONG_STAGE_BUFS 1
 #endif
+#ifdef SONG_DIST_TEAM
+constexpr bool kDistTeam = true;   // row-team distance path (query in shared memory)
+#else
+constexpr bool kDistTeam = false;  // lane-slice distance path (query in registers)
+#endif
 template <int NCH>
 struct StageRows {  // rows per round: min(SONG_STAGE_ROWS, 32 / NCH), >= 4
   static constexpr int R = (NCH >= 8) ? 4 : ((32 / NCH) < SONG_STAGE_ROWS ? (32 / NCH) : SONG_STAGE_ROWS);
@@ -765,6 +770,107 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
   return mine;
 }
 
+// Bulk distance, row-team layout (default).  A round stages R rows; each row
+// is owned by a team of LPR = 32 / R consecutive lanes and lane g of the team
+// copies (cp.async) AND later reads exactly chunks g, g + LPR, g + 2 LPR ... of
+// that row, so no lane ever reads another lane's copy (no warp barrier between
+// copy and compute), one row address per lane replaces a SHFL + IMAD per row,
+// and the reduction is log2(LPR) shuffles instead of a transposed butterfly.
+// The query sits in shared memory (qsm, 16 B chunks, zero past dpad) and is
+// read with LPR-way broadcast.  Chunk ch of row r is stored at ch ^ swz(r)
+// (rows r and r + 1 of an 8-lane LDS.128 phase land in opposite 64 B halves),
+// so both the copies and the reads are bank-conflict free.
+template <int NCH>
+struct Team {
+  static constexpr int R = StageRows<NCH>::R;  // rows per round
+  static constexpr int LPR = 32 / R;           // lanes per row
+  static constexpr int CPL = 32 * NCH / LPR;   // chunks per lane
+  __device__ __forceinline__ static int swz(int r) { return LPR == 4 ? ((r & 1) << 2) : 0; }
+};
+
+template <int NCH, int METRIC>
+__device__ __forceinline__ float bulk_distance_team(const float* __restrict__ data, int dpad,
+                                                    const int* cid, int nc, const float* qsm,
+                                                    float* stage, int cosine, int lane) {
+  using T = Team<NCH>;
+  constexpr int R = T::R, LPR = T::LPR, CPL = T::CPL;
+  constexpr int SR = Stage<NCH>::STRIDE;  // floats per staged row
+  const int d4 = dpad >> 2;
+  const int r = lane / LPR;  // row of this lane within a round
+  const int g = lane % LPR;  // chunk phase of this lane
+  const int sw = T::swz(r);
+  const int myc = d4 > g ? (d4 - g + LPR - 1) / LPR : 0;  // my chunks inside the row
+  const bool full = myc >= CPL;
+  const uint32_t rowbytes = 4u * (uint32_t)dpad;
+  const uint32_t st_row = smem_u32(stage) + (uint32_t)(r * SR * 4);
+  const float4* q4 = reinterpret_cast<const float4*>(qsm);
+  const float4* srow = reinterpret_cast<const float4*>(stage + r * SR);
+  constexpr int NBUF = StageRows<NCH>::NBUF;  // rounds in flight
+  const int rounds = (nc + R - 1) / R;
+  float mine = 0.0f;
+  // ---- copy: this lane's chunks of row k*R + r into stage buffer k % NBUF
+  auto issue = [&](int k) {
+    const int j = k * R + r;
+    if (j < nc) {
+      const char* src = reinterpret_cast<const char*>(data) + (uint64_t)(uint32_t)cid[j] * rowbytes;
+      const uint32_t dst = st_row + (uint32_t)((k % NBUF) * R * SR * 4);
+#pragma unroll
+      for (int c = 0; c < CPL; ++c) {
+        const int ch = g + LPR * c;
+        if (full || c < myc)
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + (uint32_t)((ch ^ sw) * 16)),
+                       "l"(src + ch * 16)
+                       : "memory");
+      }
+    }
+    cp_async_commit();
+  };
+  for (int k = 0; k < NBUF && k < rounds; ++k) issue(k);
+  for (int k = 0; k < rounds; ++k) {
+    const int j = k * R + r;
+    cp_async_wait_pending(min(NBUF - 1, rounds - 1 - k));
+    // ---- compute: the same chunks, read back by the lane that copied them
+    const float4* buf = srow + (size_t)(k % NBUF) * R * SR / 4;
+    float part = 0.0f;
+    if (j < nc) {
+      uint64_t acc = 0;
+#pragma unroll 8
+      for (int c = 0; c < CPL; ++c) {
+        const int ch = g + LPR * c;
+        const float4 x = buf[ch ^ sw];  // (chunks past dpad hold 0, like the query)
+        const float4 qq = q4[ch];
+        const uint64_t q01 = f2pack(qq.x, qq.y), q23 = f2pack(qq.z, qq.w);
+        acc = (c == 0) ? acc4_first<METRIC>(q01, q23, x) : acc4<METRIC>(acc, q01, q23, x);
+      }
+      part = f2sum(acc);
+    }
+    if (k + NBUF < rounds) issue(k + NBUF);  // (this lane read only its own chunks)
+#pragma unroll
+    for (int o = 1; o < LPR; o <<= 1) part += __shfl_xor_sync(FULL, part, o);
+    const int b = k * R;
+    const float got = __shfl_sync(FULL, part, ((lane - b) & (R - 1)) * LPR);
+    if (lane >= b && lane < b + R) mine = got;
+  }
+  if (METRIC == MET_DOT) mine = cosine ? 1.0f - mine : -mine;  // 1 - cos / -<q,x>
+  return mine;
+}
+
+// the distance stage used by the kernel: codes -> Hamming; float rows -> the
+// lane-slice + transposed butterfly path, or the row-team path with
+// SONG_DIST_TEAM (fewer instructions, but measured slower at 1 buffer: see
+// profiles/r01_history.md)
+template <int NCH, int METRIC>
+__device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpad, const int* cid,
+                                         int nc, const float4 (&qv)[NCH], const float* qsm,
+                                         float* stage, int cosine, int lane) {
+#ifndef SONG_DIST_TEAM
+  return bulk_distance<NCH, METRIC>(data, dpad, cid, nc, qv, stage, cosine, lane);
+#else
+  if constexpr (METRIC == MET_HAM) return hamming_distance<NCH>(data, dpad, cid, nc, qv, lane);
+  return bulk_distance_team<NCH, METRIC>(data, dpad, cid, nc, qsm, stage, cosine, lane);
+#endif
+}
+
 // ---------------------------------------------------------- the kernel --
 #ifndef SONG_LB_THREADS
 #define SONG_LB_THREADS 128
@@ -794,7 +900,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
   float* stage = reinterpret_cast<float*>(base);                       // staged rows
   const size_t stage_bytes =  // (Hamming codes are gathered straight into registers)
       METRIC == MET_HAM ? 0 : (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
-  int* cid = reinterpret_cast<int*>(base + stage_bytes + 16);
+  // the query, 16 B chunks (row-team distance path)
+  float* qsm = reinterpret_cast<float*>(base + stage_bytes);
+  constexpr size_t qsm_bytes = (METRIC == MET_HAM || !kDistTeam) ? 0 : (size_t)NCH * 512;
+  int* cid = reinterpret_cast<int*>(base + stage_bytes + qsm_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + (MS ? 32 * MAX_STEPS : 32));  // 32 keys
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
   uint64_t* qa = ev + 32;                                               // QR == 0 only
@@ -897,6 +1006,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         qv[c].w *= inv;
       }
     }
+    if constexpr (METRIC != MET_HAM && kDistTeam) {
+      // stage the (normalised) query in shared memory: chunk c*32 + lane
+      __syncwarp();
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) reinterpret_cast<float4*>(qsm)[c * 32 + lane] = qv[c];
+      __syncwarp();
+    }
     int32_t* ids_o = a.ids_out + (int64_t)qi * a.K;
     float* dists_o = a.dists_out + (int64_t)qi * a.K;
     if (bad) {
@@ -917,7 +1033,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
     if (VK == VK_GHASH) gh.gen = ++gen;  // a fresh generation empties the table
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    const float de = bulk_distance<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, stage, a.cosine, lane);
+    const float de = dist_of<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, qsm, stage, a.cosine, lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     v_insert_lane0(a.entry);
     int used = 1;  // VK_HASH: live + tombstones; VK_GHASH: live
@@ -1076,7 +1192,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
 
       // ---- a5: bulk distance computation (§VI)
       const float dist =
-          bulk_distance<NCH, METRIC>(a.data, a.dpad, cidg, nc, qv, stage, a.cosine, lane);
+          dist_of<NCH, METRIC>(a.data, a.dpad, cidg, nc, qv, qsm, stage, a.cosine, lane);
 
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cidg[lane] : -1;

@@ -198,7 +198,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     s.lazy = p->visited_cap >= 0 && p->steps <= 1;
     if (s.lazy)
       s.rebuild_at = p->visited_cap > 0 ? p->visited_cap
-                                        : (big ? (3 << s.table_log2) / 4 : (1 << s.table_log2) / 2);
+                                        : (big ? (3 << s.table_log2) / 4 : (5 << s.table_log2) / 8);
     tbytes = (1 << s.table_log2) * 4;
   }
   // float rows: NCH = 16 B chunks per lane (128 floats per chunk row);
@@ -209,7 +209,8 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
-  s.warp_bytes = stage_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
+  const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
+  s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
                  (s.qr == 0 ? 3 * L * 8 + 8 : 0) + tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   return s;

@@ -323,7 +323,7 @@ def default_visited_cap(L: int) -> int:
     slots = 1
     while slots < need:
         slots <<= 1
-    return 3 * slots // 4 if big else slots // 2
+    return 3 * slots // 4 if big else 5 * slots // 8
 
 
 def rp_encode(vectors, R):
