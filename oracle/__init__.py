@@ -6,7 +6,7 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R14 it follows are listed in its header and in DESIGN.md §3).
+R1-R15 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
@@ -89,6 +89,9 @@ def _load():
         lib.oracle_rp_encode.restype = None
         lib.oracle_rp_encode.argtypes = [P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, P,
                                          ctypes.c_int32]
+        lib.oracle_build_graph.restype = None
+        lib.oracle_build_graph.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                           ctypes.c_int32, P, ctypes.c_int32]
         lib.oracle_bloom_probe.restype = None
         lib.oracle_bloom_probe.argtypes = [ctypes.c_int64, P, ctypes.c_int64, P,
                                            ctypes.c_int64, P]
@@ -247,6 +250,18 @@ def hamming(a, b) -> int:
 def code_bytes(n: int, h: int) -> int:
     """Table IV: an h-bit code takes h/32 words = h/8 bytes per point."""
     return n * h // 8
+
+
+def build_graph(data, degree: int, metric: int = L2, nthreads: int = 1):
+    """Graph construction of reading R15 (exact-insertion NSW forward lists,
+    capped backward lists, HNSW heuristic with refill): adjacency [n, degree]
+    int32, -1 padded."""
+    lib = _load()
+    data = _f32(data)
+    n, dim = data.shape
+    adj = np.empty((n, degree), np.int32)
+    lib.oracle_build_graph(_ptr(data), n, dim, metric, degree, _ptr(adj), int(nthreads))
+    return adj
 
 
 def recall(found_ids, truth_ids) -> float:

@@ -51,6 +51,17 @@
 //      evicted from q ∪ topk has L better vertices there for good), so only
 //      the counters move: fewer recomputed distances than eager deletion,
 //      memory still bounded by C >= 2L + 32.
+//   R15 graph construction (the step before the search: SONG loads NSW graphs,
+//      P:477; HNSW layer-0 style): with every distance the search's
+//      own (R7) and every order the (dist, id) key (R2), degree D:
+//      1. forward F(i) = the D smallest keys (d(i, j), j) over j < i
+//         (exact-insertion NSW: each vertex links to its D nearest earlier ones);
+//      2. backward B(j) = the D smallest keys (d(i, j), i) over {i : j in F(i)};
+//      3. C(v) = F(v) u B(v) (disjoint: ids < v and > v) ascending by key;
+//      4. HNSW heuristic: walk C(v) in order, keep c while fewer than D are kept
+//         and d(c, k) > d(c, v) for every kept k ("closer to the base than to
+//         every kept neighbour"); then refill with the skipped candidates in
+//         C(v) order up to D; pad with -1.  Row = kept then refilled, in order.
 //   R12 Hamming search: the distance of two codes is the number of differing
 //      bits ("the hamming distance between the bit-vectors"), used as the
 //      key's distance (an integer, exact in fp32) with the same (dist, id)
@@ -536,6 +547,72 @@ void oracle_rp_encode(const float* data, int64_t n, int32_t dim, const float* R,
       for (int64_t i = t; i < n; i += nthreads) one(i);
     });
   for (auto& th : pool) th.join();
+}
+
+// R15: graph construction (see the header).  data [n][dim] fp32, adj_out
+// [n][degree] int32.  nthreads > 1 splits the per-vertex loops over threads.
+void oracle_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t degree,
+                        int32_t* adj_out, int32_t nthreads) {
+  const int D = degree;
+  auto dist = [&](int64_t a, int64_t b) {
+    return distance(data + a * dim, data + b * dim, dim, metric);
+  };
+  auto parallel = [&](auto&& fn) {
+    if (nthreads <= 1) {
+      for (int64_t v = 0; v < n; ++v) fn(v);
+      return;
+    }
+    std::vector<std::thread> pool;
+    for (int t = 0; t < nthreads; ++t)
+      pool.emplace_back([&, t]() {
+        for (int64_t v = t; v < n; v += nthreads) fn(v);
+      });
+    for (auto& th : pool) th.join();
+  };
+  // 1. forward lists
+  std::vector<std::vector<Key>> F(n);
+  parallel([&](int64_t i) {
+    std::vector<Key> all;
+    all.reserve(i);
+    for (int64_t j = 0; j < i; ++j) all.push_back(Key{dist(i, j), (int32_t)j});
+    const size_t k = std::min<size_t>(D, all.size());
+    std::partial_sort(all.begin(), all.begin() + k, all.end());
+    all.resize(k);
+    F[i] = all;
+  });
+  // 2. backward lists
+  std::vector<std::vector<Key>> B(n);
+  for (int64_t i = 0; i < n; ++i)
+    for (const Key& e : F[i]) B[e.id].push_back(Key{e.dist, (int32_t)i});
+  parallel([&](int64_t j) {
+    auto& b = B[j];
+    const size_t k = std::min<size_t>(D, b.size());
+    std::partial_sort(b.begin(), b.begin() + k, b.end());
+    b.resize(k);
+  });
+  // 3. + 4. candidates and the heuristic
+  parallel([&](int64_t v) {
+    std::vector<Key> C = F[v];
+    C.insert(C.end(), B[v].begin(), B[v].end());
+    std::sort(C.begin(), C.end());
+    std::vector<int32_t> kept;
+    std::vector<char> taken(C.size(), 0);
+    for (size_t t = 0; t < C.size() && (int)kept.size() < D; ++t) {
+      bool ok = true;
+      for (int32_t k : kept)
+        if (!(dist(C[t].id, k) > C[t].dist)) {
+          ok = false;
+          break;
+        }
+      if (ok) {
+        kept.push_back(C[t].id);
+        taken[t] = 1;
+      }
+    }
+    for (size_t t = 0; t < C.size() && (int)kept.size() < D; ++t)
+      if (!taken[t]) kept.push_back(C[t].id);
+    for (int j = 0; j < D; ++j) adj_out[v * D + j] = j < (int)kept.size() ? kept[j] : -1;
+  });
 }
 
 // Cuckoo filter probe for tests of R10: applies ops[i] (+id = insert,
