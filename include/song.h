@@ -244,6 +244,20 @@ int song_search_codes_ex(song_index* idx, const song_search_params* params,
                          const uint32_t* query_codes, int64_t nq, int32_t* ids_out,
                          float* dists_out, int32_t* counters_out, void* stream);
 
+/* ---- graph construction (reading R15) ----
+ * SONG searches pre-built NSW graphs; this builds one on the
+ * device: forward lists F(i) = the `degree` nearest earlier vertices (exact
+ * insertion NSW), backward lists B(j) = the `degree` nearest i with j in F(i),
+ * candidates F(v) u B(v) by (dist, id), HNSW neighbour heuristic with refill,
+ * -1 padding.  Distances are the search's (L2 squared, -<a,b>, 1 - cos).
+ *   vectors       DEVICE [n][dim] fp32 (not modified)
+ *   adjacency_out DEVICE [n][degree] int32 (caller-allocated)
+ * Blocking on stream (scratch ~ 24 n degree bytes is allocated and freed).
+ * Errors: SONG_EINVAL (NULL, sizes < 1, metric), SONG_EUNSUPPORTED (degree >
+ * SONG_MAX_DEGREE, n >= 2^31), SONG_ENOMEM, SONG_ECUDA. */
+int song_build_graph(const float* vectors, int64_t n, int32_t dim, song_metric metric,
+                     int32_t degree, int32_t* adjacency_out, void* stream);
+
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);
 

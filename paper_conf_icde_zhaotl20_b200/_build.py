@@ -14,7 +14,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libsong.so")
-SOURCES = ["song_api.cu", "launch_nch1.cu", "launch_nch2.cu", "launch_nch4.cu", "launch_nch8.cu"]
+SOURCES = ["song_api.cu", "launch_nch1.cu", "launch_nch2.cu", "launch_nch4.cu", "launch_nch8.cu",
+           "graph_build.cu"]
 DEPS = [os.path.join(CSRC, f) for f in os.listdir(CSRC)] + [os.path.join(ROOT, "include", "song.h")]
 
 NVCC_FLAGS = [

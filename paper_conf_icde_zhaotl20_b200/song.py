@@ -33,7 +33,7 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
-            "song_search_codes_ex"]
+            "song_search_codes_ex", "song_build_graph"]
 
 
 class SongError(RuntimeError):
@@ -86,6 +86,7 @@ def lib():
         L.song_index_create_codes.argtypes = [P, i64, i32, P, i32, PP]
         L.song_index_create_rp.argtypes = [P, i64, i32, P, i32, P, i32, PP]
         L.song_search_codes_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
+        L.song_build_graph.argtypes = [P, i64, i32, i32, i32, P, P]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -94,7 +95,7 @@ def lib():
                      "song_index_get_info", "song_search", "song_search_ex",
                      "song_index_last_status", "song_merge_topk", "song_rp_encode",
                      "song_index_create_codes", "song_index_create_rp",
-                     "song_search_codes_ex"):
+                     "song_search_codes_ex", "song_build_graph"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -314,6 +315,22 @@ def merge_topk(ids, dists, K: int):
                                  G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
                                  ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
     return oi, od
+
+
+def build_graph(vectors, degree: int = 32, metric: str = "l2"):
+    """song_build_graph: CUDA tensor vectors [n, dim] -> adjacency [n, degree]
+    int32 CUDA tensor (NSW forward lists + backward lists + HNSW heuristic,
+    DESIGN.md reading R15)."""
+    torch = _torch()
+    if not _is_cuda_tensor(vectors):
+        raise TypeError("build_graph() takes a CUDA tensor")
+    v = vectors.contiguous().float()
+    adj = torch.empty((v.shape[0], degree), dtype=torch.int32, device=v.device)
+    with torch.cuda.device(v.device):
+        _check(lib().song_build_graph(ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1],
+                                      METRICS[metric], degree, ctypes.c_void_p(adj.data_ptr()),
+                                      _stream_ptr(v.device)))
+    return adj
 
 
 def default_visited_cap(L: int) -> int:
