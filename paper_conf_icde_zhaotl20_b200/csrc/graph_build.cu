@@ -3,10 +3,14 @@
 #include <cuda_runtime.h>
 
 #include <cub/device/device_scan.cuh>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 #include "graph_kernel.cuh"
+#include "knn_tc.cuh"
 #include "song.h"
 #include "song_internal.h"
 
@@ -47,6 +51,28 @@ __global__ void narrow_kernel(const unsigned long long* a, int* b, int64_t n) {
        i += (int64_t)gridDim.x * blockDim.x)
     b[i] = (int)a[i];
 }
+// TMA descriptor of X [n][dim] fp32: 32-float x 128-row boxes, SWIZZLE_128B
+// (the layout the UMMA descriptors of knn_tc.cuh expect)
+int make_xmap(CUtensorMap* map, const float* x, int64_t n, int dim) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", reinterpret_cast<void**>(&encode),
+                                cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !encode)
+      return fail(SONG_ECUDA, "cuTensorMapEncodeTiled is unavailable");
+  }
+  cuuint64_t dims[2] = {(cuuint64_t)dim, (cuuint64_t)n};
+  cuuint64_t strides[1] = {(cuuint64_t)dim * 4};
+  cuuint32_t box[2] = {(cuuint32_t)song::graph::tc::TK, (cuuint32_t)song::graph::tc::TM};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(x), dims,
+                      strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(SONG_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return SONG_OK;
+}
 }  // namespace
 
 #define G_TRY(expr)                                                                   \
@@ -78,7 +104,8 @@ extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, so
   unsigned long long* cnt = nullptr;
   int64_t* off = nullptr;
   int *cursor = nullptr, *cnt32 = nullptr;
-  G_TRY(s.get(&norms, n * sizeof(float)));
+  G_TRY(s.get(&norms, (n + 256) * sizeof(float)));  // (+ tail: tile-wide norm loads)
+  G_TRY(cudaMemsetAsync(norms, 0, (n + 256) * sizeof(float), st));
   const float* x = vectors;
   if (metric == SONG_COSINE) {  // normalise a scratch copy (1 - cos)
     G_TRY(s.get(&xs, (size_t)n * dim * sizeof(float)));
@@ -97,10 +124,39 @@ extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, so
   row_norms_kernel<<<blocks, 256, 0, st>>>(const_cast<float*>(x), n, dim, norms,
                                            metric == SONG_COSINE);
   G_TRY(cudaGetLastError());
-  // 1. forward lists
-  const int64_t nb = (n + BM - 1) / BM;
-  knn_prefix_kernel<<<(unsigned)nb, THREADS, 0, st>>>(x, n, dim, norms, met, D, fkeys);
-  G_TRY(cudaGetLastError());
+  // 1. forward lists: tensor cores (tcgen05, tf32) when that is exact for the
+  // data (every value tf32-representable, rows 16 B aligned), else fp32 FFMA
+  bool use_tc = dim % 4 == 0 && metric != SONG_COSINE;
+  const char* force = std::getenv("SONG_GRAPH_PATH");  // "simt" / "tc" (tests, A/B)
+  if (use_tc && !(force && std::strcmp(force, "tc") == 0)) {
+    int* d_flag = nullptr;
+    G_TRY(s.get(&d_flag, sizeof(int)));
+    G_TRY(cudaMemsetAsync(d_flag, 0, sizeof(int), st));
+    song::graph::tc::tf32_exact_kernel<<<592, 256, 0, st>>>(x, n * (int64_t)dim, d_flag);
+    G_TRY(cudaGetLastError());
+    int not_exact = 0;
+    G_TRY(cudaMemcpyAsync(&not_exact, d_flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+    G_TRY(cudaStreamSynchronize(st));
+    use_tc = !not_exact;
+  }
+  if (force && std::strcmp(force, "simt") == 0) use_tc = false;
+  if (use_tc) {
+    namespace tc = song::graph::tc;
+    CUtensorMap xmap;
+    int rc = make_xmap(&xmap, x, n, dim);
+    if (rc) return rc;
+    G_TRY(cudaFuncSetAttribute(tc::knn_prefix_tc_kernel,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               (int)tc::SMEM_BYTES));
+    const int64_t nbt = (n + tc::TM - 1) / tc::TM;
+    tc::knn_prefix_tc_kernel<<<(unsigned)nbt, tc::THREADS, tc::SMEM_BYTES, st>>>(
+        xmap, n, dim, norms, met, D, fkeys);
+    G_TRY(cudaGetLastError());
+  } else {
+    const int64_t nb = (n + BM - 1) / BM;
+    knn_prefix_kernel<<<(unsigned)nb, THREADS, 0, st>>>(x, n, dim, norms, met, D, fkeys);
+    G_TRY(cudaGetLastError());
+  }
   // 2. backward lists
   G_TRY(cudaMemsetAsync(cnt, 0, n * sizeof(unsigned long long), st));
   G_TRY(cudaMemsetAsync(cursor, 0, n * sizeof(int), st));

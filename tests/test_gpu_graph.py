@@ -31,20 +31,35 @@ def test_toy():
     np.testing.assert_array_equal(gbuild(x, 2), want)
 
 
-@pytest.mark.parametrize("n,dim,D", [(1, 3, 4), (2, 3, 4), (63, 5, 4), (64, 5, 8), (65, 7, 8),
-                                     (300, 3, 16), (1000, 30, 32), (777, 130, 12)])
-def test_integer_random_bit_exact(n, dim, D):
-    """ragged n (tile tails), ragged dims (k tails), many exact ties."""
+@pytest.mark.parametrize("path", ["auto", "simt", "tc"])
+@pytest.mark.parametrize("n,dim,D", [(1, 4, 4), (2, 4, 4), (63, 8, 4), (64, 8, 8), (65, 12, 8),
+                                     (127, 4, 16), (129, 36, 16), (300, 4, 16), (1000, 32, 32),
+                                     (777, 132, 12), (2100, 64, 32)])
+def test_integer_random_bit_exact(n, dim, D, path, monkeypatch):
+    """ragged n (tile tails: 64-row SIMT tiles, 128-row tensor-core tiles),
+    ragged dims (k tails), many exact ties; both forward-list paths (the
+    tensor-core path is exact on these tf32-representable integers)."""
+    if path != "auto":
+        monkeypatch.setenv("SONG_GRAPH_PATH", path)
     rng = np.random.default_rng(n + dim + D)
     x = rng.integers(0, 12, (n, dim)).astype(np.float32)
     np.testing.assert_array_equal(gbuild(x, D), oracle.build_graph(x, D, nthreads=8))
 
 
-def test_sift_shaped_bit_exact():
+@pytest.mark.parametrize("path", ["tc", "simt"])
+def test_sift_shaped_bit_exact(path, monkeypatch):
+    monkeypatch.setenv("SONG_GRAPH_PATH", path)
     cfg = CONFIGS["sift1m"]
     x, _ = make_data(cfg, n=6000, nq=1)
     xn = x.numpy()
     np.testing.assert_array_equal(gbuild(xn, 32), oracle.build_graph(xn, 32, nthreads=8))
+
+
+def test_odd_dims_take_the_simt_path():
+    """dim % 4 != 0 (no 16 B TMA rows) and non-tf32 values use fp32 FFMA tiles."""
+    rng = np.random.default_rng(1)
+    x = rng.integers(0, 9, (500, 7)).astype(np.float32)
+    np.testing.assert_array_equal(gbuild(x, 8), oracle.build_graph(x, 8))
 
 
 @pytest.mark.parametrize("metric", ["l2", "ip", "cosine"])
