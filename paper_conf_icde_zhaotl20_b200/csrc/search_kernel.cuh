@@ -532,6 +532,9 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
 #ifndef SONG_STAGE_ROWS
 #define SONG_STAGE_ROWS 8
 #endif
+#ifndef SONG_L2_PREFETCH
+#define SONG_L2_PREFETCH 2
+#endif
 #ifndef SONG_STAGE_BUFS
 #define SONG_STAGE_BUFS 1
 #endif
@@ -736,6 +739,20 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     cp_async_commit();
   };
   for (int k = 0; k < NBUF && k < rounds; ++k) issue(k);
+#if SONG_L2_PREFETCH
+  // rows of the later rounds start their DRAM trip now: each such lane asks
+  // L2 for its own candidate's row, so round k >= NBUF waits on an L2 hit
+  // instead of a second dependent DRAM round trip
+  if (lane >= NBUF * R && lane < nc) {
+    const char* row = reinterpret_cast<const char*>(data) + (uint64_t)myid * rowbytes;
+#if SONG_L2_PREFETCH == 1
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(row), "r"(rowbytes) : "memory");
+#else
+    for (uint32_t o = 0; o < rowbytes; o += 128)
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(row + o));
+#endif
+  }
+#endif
   for (int k = 0; k < rounds; ++k) {
     const int b = k * R;
     const int rows = min(R, nc - b);
