@@ -106,7 +106,7 @@ typedef struct song_search_params {
   int32_t visited_cap;     /* SONG_VISITED_HASH deletion schedule (§IV-E, DESIGN.md
                               reading R14).  0 = lazy deletion with the default capacity
                               C = 5S/8 for queue_len <= 128, 3S/4 above, where S =
-                              2^ceil(log2(F (2L + 32))) table slots, F = 8 (L <= 128) or
+                              2^ceil(log2(F (2L + 32))) table slots, F = 8 (L <= 64), 4 (L <= 128) or
                               2; > 0 = lazy with C = visited_cap (2L + 32 <= C <= 3S/4,
                               else SONG_EINVAL); -1 = eager deletion (every evicted vertex
                               erased at once, the paper's literal schedule).  Lazy: the

@@ -157,6 +157,9 @@ int check_create_args(const void* vectors, int64_t n, int32_t dim, const void* a
 #ifndef SONG_HASH_FACTOR
 #define SONG_HASH_FACTOR 8
 #endif
+#ifndef SONG_HASH_FACTOR_WIDE  // 64 < L <= 128 (QR = 4)
+#define SONG_HASH_FACTOR_WIDE 4
+#endif
 #ifndef SONG_HASH_REBUILD_NUM  // rebuild at NUM/16 occupancy
 #define SONG_HASH_REBUILD_NUM 4
 #endif
@@ -169,6 +172,12 @@ struct Shape {
   int qr;  // register queue width (L <= 32*qr), 0 = shared-memory queues
   int nch;
 };
+
+// slots of the shared-memory visited hash: >= F (2L + 32), the live-key bound
+int hash_log2_slots(int L) {
+  const long long F = L > 128 ? 2 : L > 64 ? SONG_HASH_FACTOR_WIDE : SONG_HASH_FACTOR;
+  return next_pow2_log2(F * (2ll * L + 32));
+}
 
 Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
   const int steps = p->steps;
@@ -188,11 +197,12 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     tbytes = (4 << s.table_log2) * 2;
   } else {
     // live keys <= |q| + |topk| + 32 new ones <= 2L + 32.  Register-queue
-    // sizes get >= 8x that many slots and rebuild at 1/4 occupancy (about one
+    // sizes get >= 8x (L <= 64) or 4x (L <= 128: a 16 KB table would cut
+    // residency to 10 warps/SM, measured 2.7M -> 3.9M QPS at K = 100) that many slots and rebuild at 1/4 occupancy (about one
     // probe per operation); shared-memory queues (L > 128) get >= 2x and
     // rebuild at 3/4 to bound shared memory.
     const bool big = L > 128;
-    s.table_log2 = next_pow2_log2((big ? 2ll : (long long)SONG_HASH_FACTOR) * (2 * L + 32));
+    s.table_log2 = hash_log2_slots(L);
     s.rebuild_at = big ? (3 << s.table_log2) / 4 : (SONG_HASH_REBUILD_NUM << s.table_log2) / 16;
     // lazy deletion (R14): visited holds up to C live ids, no tombstones
     s.lazy = p->visited_cap >= 0 && p->steps <= 1;
@@ -236,8 +246,7 @@ int check_params(const song_index* ix, const song_search_params* p) {
   if (p->visited_cap < -1) return fail(SONG_EINVAL, "visited_cap %d < -1", p->visited_cap);
   if (p->visited_cap > 0 && p->visited == SONG_VISITED_HASH) {
     const bool big = p->queue_len > 128;
-    const int slots = 1 << next_pow2_log2((big ? 2ll : (long long)SONG_HASH_FACTOR) *
-                                          (2ll * p->queue_len + 32));
+    const int slots = 1 << hash_log2_slots(p->queue_len);
     if (p->visited_cap < 2 * p->queue_len + 32 || p->visited_cap > 3 * (slots / 4))
       return fail(SONG_EINVAL, "visited_cap %d outside [2L + 32, 3/4 of %d slots]",
                   p->visited_cap, slots);

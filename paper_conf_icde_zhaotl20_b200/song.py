@@ -336,7 +336,7 @@ def build_graph(vectors, degree: int = 32, metric: str = "l2"):
 def default_visited_cap(L: int) -> int:
     """The default lazy-deletion capacity C of include/song.h (visited_cap = 0)."""
     big = L > 128
-    need = (2 if big else 8) * (2 * L + 32)
+    need = (2 if big else 4 if L > 64 else 8) * (2 * L + 32)
     slots = 1
     while slots < need:
         slots <<= 1

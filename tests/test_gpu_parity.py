@@ -34,9 +34,9 @@ ALL_VISITED = list(ORACLE_FLAGS)
 
 def lazy_cap_for(L):
     """include/song.h's default lazy-deletion capacity (visited_cap = 0):
-    5S/8 for L <= 128, 3S/4 above, S = 2^ceil(log2(F (2L + 32))), F = 8 or 2."""
+    5S/8 for L <= 128, 3S/4 above, S = 2^ceil(log2(F (2L + 32))), F = 8 (L <= 64), 4 (L <= 128) or 2."""
     big = L > 128
-    slots = 1 << int(np.ceil(np.log2((2 if big else 8) * (2 * L + 32))))
+    slots = 1 << int(np.ceil(np.log2((2 if big else 4 if L > 64 else 8) * (2 * L + 32))))
     return 3 * slots // 4 if big else 5 * slots // 8
 
 

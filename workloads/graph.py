@@ -99,8 +99,10 @@ def _heuristic_prune(x, cand, cand_d, degree, metric, block):
 
 def build_graph(x: torch.Tensor, degree: int = 32, metric: str = "l2", M: int = None,
                 rev_cap: int = None, row_block: int = 8192, col_block: int = 65536,
-                prune_block: int = 8192) -> torch.Tensor:
-    """Returns int32 adjacency [n, degree] (-1 padded) on x's device."""
+                prune_block: int = 8192, heuristic: bool = True) -> torch.Tensor:
+    """Returns int32 adjacency [n, degree] (-1 padded) on x's device.
+    heuristic=False keeps the `degree` nearest of F(v) u B(v) (plain NSW lists,
+    probe only: reading R15 always applies the heuristic)."""
     x = x.float()
     if metric == "cosine":
         x = x / x.norm(dim=1, keepdim=True).clamp_min(1e-30)
@@ -133,5 +135,7 @@ def build_graph(x: torch.Tensor, degree: int = 32, metric: str = "l2", M: int = 
     srt = torch.sort(cand_d, dim=1, stable=True).indices
     cand = torch.gather(cand, 1, srt)
     cand_d = torch.gather(cand_d, 1, srt)
+    if not heuristic:
+        return cand[:, :degree].to(torch.int32)
     adj = _heuristic_prune(x, cand, cand_d, degree, metric, prune_block)
     return adj.to(torch.int32)
