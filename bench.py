@@ -380,13 +380,17 @@ def run_song(args, ws, rank, local, log):
             "kernel": kernel_name(cfg, L_op, args.visited), "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "n_dist": n_dist, "n_exp": n_exp,
             "kernel_ms": round(kernel_s * 1e3, 4),
+            "kernel_ms_note": "whole step on the launching stream: search kernel + outlier-first scheduling kernels (conservative for the search kernel alone)",
         },
         "e2e": {"value": round(e2e_value, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(qh.numel() * 4),
                 "d2h_bytes_per_step": int(ih.numel() * 4 + dh.numel() * 4),
                 "host_results_match_device": host_ok},
         "clocks": clk.summary(),
-        "gpu_launches": args.steps,
+        # per step: the search kernel, plus the two outlier-first scheduling
+        # kernels (order keys + scatter) when the batch outnumbers the resident
+        # warps (song.h SONG_SCHEDULE_AUTO)
+        "gpu_launches": args.steps * (3 if nq > 24 * torch.cuda.get_device_properties(dev).multi_processor_count else 1),
     }
 
     # ---- CPU baseline: the oracle as it stands, bounded sample, rank 0, N=1

@@ -115,7 +115,22 @@ typedef struct song_search_params {
                               would grow visited past C — same results, fewer recomputed
                               distances.  steps > 1 always uses eager deletion.  Ignored
                               by the other visited kinds. */
+  int32_t schedule;        /* order in which the batch's queries are issued to the
+                              persistent grid (a scheduling choice: every query's ids,
+                              distances and counters are independent of it).
+                              SONG_SCHEDULE_AUTO (0, default) = outlier-first for float
+                              indexes when nq exceeds the grid's resident warps, else
+                              batch order; SONG_SCHEDULE_BATCH = batch order;
+                              SONG_SCHEDULE_OUTLIER_FIRST = descending squared distance
+                              from the index centroid (longest-expected-first list
+                              scheduling: far-out queries search longest),
+                              in 4096 log-spaced key bins.  Codes indexes always use
+                              batch order. */
 } song_search_params;
+
+#define SONG_SCHEDULE_AUTO 0
+#define SONG_SCHEDULE_BATCH 1
+#define SONG_SCHEDULE_OUTLIER_FIRST 2
 
 typedef struct song_index_info {
   int64_t n;               /* points */

@@ -56,6 +56,7 @@ struct SearchArgs {
   float* dists_out;       // [nq][K]
   int32_t* counters_out;  // [nq][2] or nullptr
   unsigned* ticket;       // work counter, zeroed before launch
+  const int32_t* order;   // [nq] ticket -> query index, or nullptr (batch order)
   int* status;            // sticky STATUS_* bits
   int64_t n;
   int64_t nq;
@@ -978,7 +979,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
   uint32_t gen = a.gen0;
   while (true) {
     int qi = 0;
-    if (lane == 0) qi = (int)atomicAdd(a.ticket, 1u);
+    if (lane == 0) {
+      qi = (int)atomicAdd(a.ticket, 1u);
+      if (a.order && (int64_t)qi < a.nq) qi = __ldg(a.order + qi);  // scheduled order
+    }
     qi = __shfl_sync(FULL, qi, 0);
     if ((int64_t)qi >= a.nq) break;
 

@@ -15,6 +15,7 @@
 
 #include "merge_kernel.cuh"
 #include "rp_kernel.cuh"
+#include "schedule.cuh"
 #include "search_kernel.cuh"
 #include "song.h"
 
@@ -133,6 +134,10 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_dists);
   cudaFree(ix->d_gtab);
   cudaFree(ix->d_R);
+  cudaFree(ix->d_centroid);
+  cudaFree(ix->d_bins);
+  cudaFree(ix->d_order);
+  cudaFree(ix->d_qbin);
   cudaFree(ix->d_qcodes);
   if (ix->stream) cudaStreamDestroy(ix->stream);
   delete ix;
@@ -251,11 +256,39 @@ int check_params(const song_index* ix, const song_search_params* p) {
       return fail(SONG_EINVAL, "visited_cap %d outside [2L + 32, 3/4 of %d slots]",
                   p->visited_cap, slots);
   }
+  if (p->schedule < SONG_SCHEDULE_AUTO || p->schedule > SONG_SCHEDULE_OUTLIER_FIRST)
+    return fail(SONG_EINVAL, "unknown schedule %d", p->schedule);
   if (p->steps > SONG_MAX_STEPS)
     return fail(SONG_EUNSUPPORTED, "steps %d > %d", p->steps, SONG_MAX_STEPS);
   if (p->steps > 1 && ((p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM) ||
                        ix->metric == SONG_HAMMING))
     return fail(SONG_EUNSUPPORTED, "multi-step probing needs visited HASH or BLOOM on a float index");
+  return SONG_OK;
+}
+
+// outlier-first ticket order of a float query batch q [nq][dim] into ix->d_order
+int prepare_order(song_index* ix, const float* q, int64_t nq, cudaStream_t st) {
+  if ((size_t)nq > ix->cap_order) {
+    CUDA_TRY(cudaStreamSynchronize(st));
+    cudaFree(ix->d_order);
+    cudaFree(ix->d_qbin);
+    ix->d_order = nullptr;
+    ix->d_qbin = nullptr;
+    ix->cap_order = 0;
+    CUDA_TRY(cudaMalloc(&ix->d_order, (size_t)nq * sizeof(int32_t)));
+    CUDA_TRY(cudaMalloc(&ix->d_qbin, (size_t)nq * sizeof(uint16_t)));
+    ix->cap_order = (size_t)nq;
+  }
+  if (!ix->d_bins) CUDA_TRY(cudaMalloc(&ix->d_bins, 2 * song::SCHED_BINS * sizeof(unsigned)));
+  CUDA_TRY(cudaMemsetAsync(ix->d_bins, 0, 2 * song::SCHED_BINS * sizeof(unsigned), st));
+  const int kb = (int)std::min<int64_t>((nq + 7) / 8, (int64_t)ix->num_sms * 8);
+  song::order_keys_kernel<<<kb, 256, 0, st>>>(q, nq, ix->dim, ix->d_centroid,
+                                              ix->metric == SONG_COSINE, ix->d_bins, ix->d_qbin);
+  CUDA_TRY(cudaGetLastError());
+  const int sb = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)ix->num_sms);
+  song::order_scatter_kernel<<<sb, 256, 0, st>>>(nq, ix->d_bins, ix->d_bins + song::SCHED_BINS,
+                                                 ix->d_qbin, ix->d_order);
+  CUDA_TRY(cudaGetLastError());
   return SONG_OK;
 }
 
@@ -269,6 +302,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.dists_out = dists;
   a.counters_out = counters;
   a.ticket = ix->d_ticket;
+  a.order = nullptr;
   a.status = ix->d_status;
   a.n = ix->n;
   a.nq = nq;
@@ -307,6 +341,17 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
     return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
                 p->queue_len, sh.warp_bytes);
   ix->last_stream = st;
+  // ticket order (song_search_params.schedule): outlier-first needs the centroid
+  // (float indexes) and pays when the batch outnumbers the resident warps
+  const bool outlier_first =
+      ix->d_centroid && nq > 1 &&
+      (p->schedule == SONG_SCHEDULE_OUTLIER_FIRST ||
+       (p->schedule == SONG_SCHEDULE_AUTO && nq > (int64_t)ix->num_sms * 24));
+  if (outlier_first) {
+    int rc = prepare_order(ix, q, nq, st);
+    if (rc) return rc;
+    a.order = ix->d_order;
+  }
   const int m = ix->metric, qr = sh.qr, bps = p->blocks_per_sm, sms = ix->num_sms;
   switch (sh.nch) {
     case 1: return launch_m<1>(ix, a, m, vk, qr, warps, bps, sms, st);
@@ -335,6 +380,19 @@ int finish_create(song_index* ix, cudaStream_t st) {
     int blocks = (int)std::min<int64_t>((ix->n + 7) / 8, 65535);
     normalize_rows_kernel<<<blocks, 256, 0, st>>>(ix->d_data, ix->n, ix->dpad);
     CUDA_TRY(cudaGetLastError());
+  }
+  if (ix->metric != SONG_HAMMING) {  // centroid for the outlier-first schedule
+    const int64_t chunk = (ix->n + song::CENTROID_BLOCKS - 1) / song::CENTROID_BLOCKS;
+    const int nparts = (int)((ix->n + chunk - 1) / chunk);
+    float* part = nullptr;
+    CUDA_TRY(cudaMalloc(&part, (size_t)nparts * ix->dpad * sizeof(float)));
+    CUDA_TRY(cudaMalloc(&ix->d_centroid, (size_t)ix->dpad * sizeof(float)));
+    song::centroid_partial_kernel<<<nparts, 128, 0, st>>>(ix->d_data, ix->n, ix->dpad, chunk, part);
+    song::centroid_final_kernel<<<1, 256, 0, st>>>(part, nparts, ix->dpad, ix->n, ix->d_centroid);
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFree(part);
+    if (e != cudaSuccess) return fail(SONG_ECUDA, "centroid: %s", cudaGetErrorString(e));
   }
   CUDA_TRY(cudaStreamSynchronize(st));
   return SONG_OK;

@@ -36,6 +36,12 @@ struct song_index {
   float* d_R = nullptr;                // [code_bits][rp_dim] random vectors
   uint32_t* d_qcodes = nullptr;        // scratch: encoded query batch
   size_t cap_qcodes = 0;
+  // outlier-first schedule (song_search_params.schedule)
+  float* d_centroid = nullptr;         // [dpad] mean of the (normalised) rows
+  unsigned* d_bins = nullptr;          // [2][SCHED_BINS] counts, cursors
+  int32_t* d_order = nullptr;          // [nq] ticket -> query
+  uint16_t* d_qbin = nullptr;          // [nq] bin of each query
+  size_t cap_order = 0;
 };
 
 namespace song {

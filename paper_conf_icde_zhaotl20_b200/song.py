@@ -42,13 +42,17 @@ class SongError(RuntimeError):
         self.code = code
 
 
+SCHEDULES = {"auto": 0, "batch": 1, "outlier_first": 2}  # song.h SONG_SCHEDULE_*
+
+
 class SearchParams(ctypes.Structure):
     _fields_ = [("K", ctypes.c_int32), ("queue_len", ctypes.c_int32),
                 ("visited", ctypes.c_int32), ("bloom_log2_bits", ctypes.c_int32),
                 ("entry", ctypes.c_int32), ("max_iters", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32),
-                ("steps", ctypes.c_int32), ("visited_cap", ctypes.c_int32)]
+                ("steps", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
+                ("schedule", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -139,6 +143,7 @@ class Params:
     table_log2: int = 0
     steps: int = 1  # multi-step probing (pops per iteration, §V)
     visited_cap: int = 0  # hash deletion schedule: 0 lazy (default cap), >0 lazy cap, -1 eager
+    schedule: str = "auto"  # ticket order: "auto" | "batch" | "outlier_first"
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -153,6 +158,7 @@ class Params:
         p.table_log2 = self.table_log2
         p.steps = self.steps
         p.visited_cap = self.visited_cap
+        p.schedule = SCHEDULES[self.schedule]
         return p
 
 

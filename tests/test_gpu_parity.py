@@ -6,6 +6,8 @@ Bars (BASELINE.json north_star):
  * float data: top-K ids identical on >= 99.5 % of queries, distances within
    rtol 1e-5 + atol 1e-5 * scale, recall within 0.002 of the oracle's.
 """
+import ctypes
+
 import numpy as np
 import pytest
 
@@ -398,3 +400,41 @@ def test_sift1m_full_size_sampled_parity():
     assert (np.diff(dd, axis=1) >= 0).all()
     assert ((ii >= 0) & (ii < cfg.n)).all()
     assert all(len(set(r)) == cfg.K for r in ii)
+
+
+@pytest.mark.parametrize("name,L", [("sift1m", 48), ("glove200", 64), ("nytimes256", 64)])
+def test_schedule_never_changes_results(name, L):
+    """The outlier-first ticket order (song_search_params.schedule) only moves
+    queries between warps: ids, distances and counters equal the batch order's
+    for every query, and the oracle's on a sample (integer data: bit-exact)."""
+    s = song()
+    cfg = CONFIGS[name]
+    x, q = make_data(cfg, device="cuda", n=50_000, nq=6000)  # > 148 x 24 resident warps
+    adj = s.build_graph(x, cfg.degree, cfg.metric)
+    idx = s.SongIndex(x, adj, metric=cfg.metric)
+    res = {}
+    for sched in ("batch", "outlier_first", "auto"):
+        ids, d, c = idx.search(q, params=s.Params(K=cfg.K, queue_len=L, schedule=sched),
+                               counters=True)
+        torch.cuda.synchronize()
+        idx.last_status()
+        res[sched] = (ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy())
+    for sched in ("outlier_first", "auto"):
+        for a, b in zip(res["batch"], res[sched]):
+            np.testing.assert_array_equal(a, b)
+    pick = np.arange(0, 6000, 40)
+    o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()[pick], cfg.K, L,
+                      metric=oracle.METRICS[cfg.metric], nthreads=8, **oracle_kw("hash", L))
+    g = tuple(r[pick] for r in res["outlier_first"])
+    if cfg.kind == "sift":
+        assert_exact(g, o)
+    else:
+        assert_close(g, o, scale=float(np.abs(o[1]).max()), id_frac=0.99)
+    p = s.Params(K=cfg.K, queue_len=L).to_c()
+    p.schedule = 7
+    out = torch.empty((1, cfg.K), dtype=torch.int32, device="cuda")
+    rc = s.lib().song_search_ex(idx._h, ctypes.byref(p), ctypes.c_void_p(q.data_ptr()), 1,
+                                ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                None, None)
+    assert rc == -1 and b"schedule" in s.lib().song_last_error()
+    idx.close()
