@@ -96,22 +96,35 @@ __global__ void __launch_bounds__(256) order_scatter_kernel(int64_t nq,
   constexpr int PER = SCHED_BINS / 256;
   const int t = threadIdx.x;
   unsigned local[PER];
+  uint4 c4[PER / 4];  // the thread's 16 counts in 4 vector loads (one round trip)
+#pragma unroll
+  for (int k = 0; k < PER / 4; ++k) c4[k] = reinterpret_cast<const uint4*>(count)[t * (PER / 4) + k];
   unsigned s = 0;
 #pragma unroll
-  for (int k = 0; k < PER; ++k) {
-    local[k] = s;
-    s += count[t * PER + k];
+  for (int k = 0; k < PER / 4; ++k) {
+    local[4 * k + 0] = s;
+    s += c4[k].x;
+    local[4 * k + 1] = s;
+    s += c4[k].y;
+    local[4 * k + 2] = s;
+    s += c4[k].z;
+    local[4 * k + 3] = s;
+    s += c4[k].w;
   }
-  part[t] = s;
+  // exclusive scan of the 256 partial sums: within warps by shuffles, then
+  // across the 8 warp totals
+  const int lane = t & 31, w = t >> 5;
+  unsigned inc = s;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const unsigned v = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc += v;
+  }
+  if (lane == 31) part[w] = inc;
   __syncthreads();
-  // inclusive scan of the 256 partial sums (Hillis-Steele)
-  for (int d = 1; d < 256; d <<= 1) {
-    const unsigned v = t >= d ? part[t - d] : 0u;
-    __syncthreads();
-    part[t] += v;
-    __syncthreads();
-  }
-  const unsigned base = t > 0 ? part[t - 1] : 0u;
+  unsigned wbase = 0;
+  for (int k = 0; k < w; ++k) wbase += part[k];
+  const unsigned base = wbase + inc - s;
 #pragma unroll
   for (int k = 0; k < PER; ++k) off[t * PER + k] = base + local[k];
   __syncthreads();

@@ -21,6 +21,8 @@ def main():
     ap.add_argument("--L", type=int, default=48)
     ap.add_argument("--out", default="gpurun_out/order_probe.json")
     ap.add_argument("--cache", default="")
+    ap.add_argument("--only", default="")
+    ap.add_argument("--schedule", default="batch")
     a = ap.parse_args()
     import numpy as np
     import torch
@@ -30,15 +32,24 @@ def main():
     dev = torch.device("cuda", 0)
     x, q0, q, adj = bench.build_workload(cfg, dev, 0, print, a.cache)
     idx = song.SongIndex(x, adj, metric=cfg.metric)
-    p = song.Params(K=cfg.K, queue_len=a.L)
+    p = song.Params(K=cfg.K, queue_len=a.L, schedule=a.schedule)
     _, _, ctr = idx.search(q, params=p, counters=True)
     keys = {"ticket": None, "n_exp": ctr[:, 1].float(), "d_entry": ((q - x[0]) ** 2).sum(1),
             "norm": (q * q).sum(1), "d_centroid": ((q - x.mean(0)) ** 2).sum(1)}
+    g = torch.Generator(device="cuda").manual_seed(5)
+    for m in (64, 256, 1024):
+        sm = x[torch.randint(0, x.shape[0], (m,), device="cuda", generator=g)]
+        d = (q * q).sum(1, keepdim=True) + (sm * sm).sum(1)[None] - 2 * q @ sm.T
+        keys[f"mean10_of_{m}"] = d.topk(min(10, m), dim=1, largest=False).values.mean(1)
+        keys[f"mean_of_{m}"] = d.mean(1)
+    rk = lambda v: torch.argsort(torch.argsort(v)).float()
+    keys["rank_centroid+mean10_256"] = rk(keys["d_centroid"]) + rk(keys["mean10_of_256"])
+    keys["d_centroid_x_mean10_256"] = keys["d_centroid"] * keys["mean10_of_256"]
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     out = (torch.empty((q.shape[0], cfg.K), dtype=torch.int32, device=dev),
            torch.empty((q.shape[0], cfg.K), dtype=torch.float32, device=dev), None)
     res = {}
-    for name, k in keys.items():
+    for name, k in [(n, keys[n]) for n in (a.only.split(",") if a.only else keys)]:
         qq = q if k is None else q[torch.argsort(k, descending=True)].contiguous()
         for _ in range(3):
             idx.search(qq, params=p, out=out)
