@@ -63,6 +63,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="song", choices=["song", "reference"])
     ap.add_argument("--config", default="sift1m")
+    ap.add_argument("--graph", default="auto", choices=GRAPH_BUILDERS,
+                    help="graph builder: batched insertion (R16) / exact insertion (R15) / "
+                         "auto = per metric (default_graph)")
     ap.add_argument("--K", type=int, default=0, help="override the config's K (e.g. 100 for SIFT1M)")
     ap.add_argument("--target-recall", type=float, default=0.95)
     ap.add_argument("--queue-len", type=int, default=0, help="skip the sweep")
@@ -192,7 +195,30 @@ def profiled_traffic(config_key: str):
 
 
 # ------------------------------------------------------------------ workload
-def build_workload(cfg, device, rank, log, cache=""):
+GRAPH_BUILDERS = ("auto", "batched", "exact")
+
+
+def default_graph(cfg):
+    """Measured per metric: batched insertion (R16) gives the
+    L2 / cosine workloads better graphs than exact insertion (SIFT1M L 48 -> 32,
+    NYTimes 768 -> 160 at recall 0.95); on the IP workload its search-built
+    forward lists cap recall near 0.90, so IP keeps exact insertion (R15)."""
+    return "exact" if cfg.metric == "ip" else "batched"
+
+
+def build_graph_for(x, cfg, graph="auto"):
+    """The bench's graph: song_build_graph_batched (reading R16; prefix 2^16
+    rows exact, batches of m/2 searched at L = 64) or song_build_graph (R15)."""
+    from paper_conf_icde_zhaotl20_b200 import song
+    if graph == "auto":
+        graph = default_graph(cfg)
+    if graph == "exact":
+        return song.build_graph(x, cfg.degree, cfg.metric)
+    return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=1 << 16, queue_len=64,
+                                    batch_shift=1)
+
+
+def build_workload(cfg, device, rank, log, cache="", graph="auto"):
     import torch
     from workloads.synth import make_data, generator_for
     if cache and os.path.exists(cache):
@@ -207,8 +233,7 @@ def build_workload(cfg, device, rank, log, cache=""):
         q = q0
     torch.cuda.synchronize()
     t1 = time.time()
-    from paper_conf_icde_zhaotl20_b200 import song
-    adj = song.build_graph(x, cfg.degree, cfg.metric)  # the device builder (reading R15)
+    adj = build_graph_for(x, cfg, graph)  # the device builders (readings R15 / R16)
     torch.cuda.synchronize()
     t2 = time.time()
     log(f"data {t1 - t0:.1f}s graph {t2 - t1:.1f}s")
@@ -260,7 +285,8 @@ def run_song(args, ws, rank, local, log):
 
     cfg = config_of(args)
     dev = torch.device("cuda", local % torch.cuda.device_count())
-    x, q0, q, adj = build_workload(cfg, dev, rank, log, args.cache)
+    graph_used = default_graph(cfg) if args.graph == "auto" else args.graph
+    x, q0, q, adj = build_workload(cfg, dev, rank, log, args.cache, graph_used)
     idx = song.SongIndex(x, adj, metric=cfg.metric)
     truth0 = ground_truth(x, q0, cfg.K, cfg.metric)
 
@@ -363,11 +389,12 @@ def run_song(args, ws, rank, local, log):
         "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-        "data": f"synthetic ({data_desc(cfg)}, seeded; graph built on device by song_build_graph)",
+        "data": f"synthetic ({data_desc(cfg)}, seeded; graph built on device by "
+                f"{'song_build_graph_batched (R16)' if graph_used == 'batched' else 'song_build_graph (R15)'})",
         "config": {
             "workload": f"{cfg.name}-shaped: {cfg.n}x{cfg.dim} fp32 {cfg.metric}, degree-{cfg.degree} "
                         f"graph, {nq} queries/GPU, K={K}, queue_len={L_op}",
-            "n": cfg.n, "dim": d, "degree": deg, "nq_per_gpu": nq, "query_replicas": reps, "K": K, "queue_len": L_op,
+            "graph": graph_used, "n": cfg.n, "dim": d, "degree": deg, "nq_per_gpu": nq, "query_replicas": reps, "K": K, "queue_len": L_op,
             f"recall_at_{K}": round(rec, 4), "recall_sweep": sweep, "visited": args.visited,
             "visited_cap": args.visited_cap or "default (lazy deletion, reading R14)",
             "l2": "flushed between timed steps (512 MiB write)",
@@ -464,7 +491,7 @@ def run_reference(args, ws, rank, local, log):
         return None
     cfg = config_of(args)
     dev = torch.device("cuda", local) if torch.cuda.is_available() else torch.device("cpu")
-    x, q0, q, adj = build_workload(cfg, dev, 0, log)
+    x, q0, q, adj = build_workload(cfg, dev, 0, log, graph=args.graph)
     truth = ground_truth(x, q0, cfg.K, cfg.metric).cpu().numpy()
     xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q0.cpu().numpy()
     cores = len(os.sched_getaffinity(0))

@@ -273,6 +273,25 @@ int song_search_codes_ex(song_index* idx, const song_search_params* params,
 int song_build_graph(const float* vectors, int64_t n, int32_t dim, song_metric metric,
                      int32_t degree, int32_t* adjacency_out, void* stream);
 
+/* ---- batched-insertion graph construction (reading R16) ----
+ * The scale-out builder (R15's exact forward lists cost O(n^2)): rows
+ * [0, prefix) get R15's exact forward lists; then, batch by batch, rows
+ * [m, m + max(1, m >> batch_shift)) search the graph G_m built (R15 steps 2-4)
+ * from the forward lists of rows [0, m) — Algorithm 1 from entry 0 with
+ * K = degree and queue_len, this library's own search — and take its top
+ * `degree` as their forward lists; the graph is R15 steps 2-4 on every row.
+ * With prefix >= n it equals song_build_graph.
+ *   vectors       DEVICE [n][dim] fp32 (not modified)
+ *   adjacency_out DEVICE [n][degree] int32 (caller-allocated; also holds G_m
+ *                 while the batches run)
+ * Blocking on stream; scratch ~ 24 n degree bytes (+ n dpad floats when dim %
+ * 4 != 0 or cosine).  Errors: as song_build_graph; SONG_EINVAL for prefix < 1,
+ * queue_len outside [degree, SONG_MAX_QUEUE_LEN], batch_shift outside [0, 16]
+ * or non-finite vectors. */
+int song_build_graph_batched(const float* vectors, int64_t n, int32_t dim, song_metric metric,
+                             int32_t degree, int32_t prefix, int32_t queue_len,
+                             int32_t batch_shift, int32_t* adjacency_out, void* stream);
+
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);
 

@@ -89,6 +89,13 @@ def _load():
         lib.oracle_rp_encode.restype = None
         lib.oracle_rp_encode.argtypes = [P, ctypes.c_int64, ctypes.c_int32, P, ctypes.c_int32, P,
                                          ctypes.c_int32]
+        lib.oracle_forward_lists.restype = None
+        lib.oracle_forward_lists.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                             ctypes.c_int32, P, P, ctypes.c_int32]
+        lib.oracle_build_graph_from_forward.restype = None
+        lib.oracle_build_graph_from_forward.argtypes = [P, ctypes.c_int64, ctypes.c_int32,
+                                                        ctypes.c_int32, ctypes.c_int32, P, P, P,
+                                                        ctypes.c_int32]
         lib.oracle_build_graph.restype = None
         lib.oracle_build_graph.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                            ctypes.c_int32, P, ctypes.c_int32]
@@ -262,6 +269,69 @@ def build_graph(data, degree: int, metric: int = L2, nthreads: int = 1):
     adj = np.empty((n, degree), np.int32)
     lib.oracle_build_graph(_ptr(data), n, dim, metric, degree, _ptr(adj), int(nthreads))
     return adj
+
+
+def forward_lists(data, degree: int, metric: int = L2, nthreads: int = 1):
+    """R15 step 1 alone: the exact-insertion forward lists F(i) = the `degree`
+    smallest (d(i, j), j), j < i, as (ids, dists) [n, degree] (-1 / +inf pad)."""
+    lib = _load()
+    data = _f32(data)
+    n, dim = data.shape
+    ids = np.empty((n, degree), np.int32)
+    dists = np.empty((n, degree), np.float32)
+    lib.oracle_forward_lists(_ptr(data), n, dim, metric, degree, _ptr(ids), _ptr(dists),
+                             int(nthreads))
+    return ids, dists
+
+
+def build_graph_from_forward(data, fwd_ids, fwd_dists, metric: int = L2, nthreads: int = 1):
+    """R15 steps 2-4 (backward lists, candidates, heuristic with refill) on the
+    given forward lists (ids / dists [n, degree], -1 padded, ascending keys)."""
+    lib = _load()
+    data = _f32(data)
+    fwd_ids = _i32(fwd_ids)
+    fwd_dists = _f32(fwd_dists)
+    n, dim = data.shape
+    degree = fwd_ids.shape[1]
+    adj = np.empty((n, degree), np.int32)
+    lib.oracle_build_graph_from_forward(_ptr(data), n, dim, metric, degree, _ptr(fwd_ids),
+                                        _ptr(fwd_dists), _ptr(adj), int(nthreads))
+    return adj
+
+
+def batch_bounds(n: int, prefix: int, batch_shift: int):
+    """Reading R16's insertion batches: [m, m + max(1, m >> batch_shift)) from
+    m = min(n, prefix) until n."""
+    m = min(n, max(1, prefix))
+    out = []
+    while m < n:
+        b = min(n - m, max(1, m >> batch_shift))
+        out.append((m, m + b))
+        m += b
+    return out
+
+
+def build_graph_batched(data, degree: int, metric: int = L2, prefix: int = 65536,
+                        queue_len: int = 64, batch_shift: int = 1, nthreads: int = 1):
+    """Reading R16, batched-insertion NSW (the scale-out builder), step by step:
+    1. F(i) for i < prefix: R15's exact forward lists;
+    2. for each batch [m, m'): G_m = R15 steps 2-4 on F of rows [0, m); every
+       i in the batch searches G_m (Algorithm 1 from entry 0, K = degree,
+       L = queue_len) and F(i) = the search's top `degree` (ids < m);
+    3. the graph = R15 steps 2-4 on all of F."""
+    data = _f32(data)
+    n = data.shape[0]
+    D = degree
+    m0 = min(n, max(1, prefix))
+    fi = np.full((n, D), -1, np.int32)
+    fd = np.full((n, D), np.inf, np.float32)
+    fi[:m0], fd[:m0] = forward_lists(data[:m0], D, metric, nthreads)
+    for m, m1 in batch_bounds(n, prefix, batch_shift):
+        g = build_graph_from_forward(data[:m], fi[:m], fd[:m], metric, nthreads)
+        ids, dists, _, _ = search(data[:m], g, data[m:m1], D, max(queue_len, D), metric=metric,
+                                  flags=OPTIMIZED, nthreads=nthreads)
+        fi[m:m1], fd[m:m1] = ids, dists
+    return build_graph_from_forward(data, fi, fd, metric, nthreads)
 
 
 def recall(found_ids, truth_ids) -> float:

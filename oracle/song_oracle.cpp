@@ -549,10 +549,11 @@ void oracle_rp_encode(const float* data, int64_t n, int32_t dim, const float* R,
   for (auto& th : pool) th.join();
 }
 
-// R15: graph construction (see the header).  data [n][dim] fp32, adj_out
-// [n][degree] int32.  nthreads > 1 splits the per-vertex loops over threads.
-void oracle_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t degree,
-                        int32_t* adj_out, int32_t nthreads) {
+// R15 steps 2-4 (backward lists, candidates, heuristic) on given forward
+// lists F (fwd_ids / fwd_dists [n][degree], -1 padded, ascending keys).
+static void build_from_forward(const float* data, int64_t n, int32_t dim, int32_t metric,
+                               int32_t degree, std::vector<std::vector<Key>>& F,
+                               int32_t* adj_out, int32_t nthreads) {
   const int D = degree;
   auto dist = [&](int64_t a, int64_t b) {
     return distance(data + a * dim, data + b * dim, dim, metric);
@@ -569,17 +570,6 @@ void oracle_build_graph(const float* data, int64_t n, int32_t dim, int32_t metri
       });
     for (auto& th : pool) th.join();
   };
-  // 1. forward lists
-  std::vector<std::vector<Key>> F(n);
-  parallel([&](int64_t i) {
-    std::vector<Key> all;
-    all.reserve(i);
-    for (int64_t j = 0; j < i; ++j) all.push_back(Key{dist(i, j), (int32_t)j});
-    const size_t k = std::min<size_t>(D, all.size());
-    std::partial_sort(all.begin(), all.begin() + k, all.end());
-    all.resize(k);
-    F[i] = all;
-  });
   // 2. backward lists
   std::vector<std::vector<Key>> B(n);
   for (int64_t i = 0; i < n; ++i)
@@ -613,6 +603,67 @@ void oracle_build_graph(const float* data, int64_t n, int32_t dim, int32_t metri
       if (!taken[t]) kept.push_back(C[t].id);
     for (int j = 0; j < D; ++j) adj_out[v * D + j] = j < (int)kept.size() ? kept[j] : -1;
   });
+}
+
+// R15 step 1: F(i) = the D smallest keys (d(i, j), j) over j < i.
+static std::vector<std::vector<Key>> forward_lists(const float* data, int64_t n, int32_t dim,
+                                                   int32_t metric, int32_t D, int32_t nthreads) {
+  std::vector<std::vector<Key>> F(n);
+  auto one = [&](int64_t i) {
+    std::vector<Key> all;
+    all.reserve(i);
+    for (int64_t j = 0; j < i; ++j)
+      all.push_back(Key{distance(data + i * dim, data + j * dim, dim, metric), (int32_t)j});
+    const size_t k = std::min<size_t>(D, all.size());
+    std::partial_sort(all.begin(), all.begin() + k, all.end());
+    all.resize(k);
+    F[i] = all;
+  };
+  if (nthreads <= 1) {
+    for (int64_t i = 0; i < n; ++i) one(i);
+  } else {
+    std::vector<std::thread> pool;
+    for (int t = 0; t < nthreads; ++t)
+      pool.emplace_back([&, t]() {
+        for (int64_t i = t; i < n; i += nthreads) one(i);
+      });
+    for (auto& th : pool) th.join();
+  }
+  return F;
+}
+
+// R15: graph construction (see the header).  data [n][dim] fp32, adj_out
+// [n][degree] int32.  nthreads > 1 splits the per-vertex loops over threads.
+void oracle_build_graph(const float* data, int64_t n, int32_t dim, int32_t metric, int32_t degree,
+                        int32_t* adj_out, int32_t nthreads) {
+  auto F = forward_lists(data, n, dim, metric, degree, nthreads);
+  build_from_forward(data, n, dim, metric, degree, F, adj_out, nthreads);
+}
+
+// R15 step 1 alone: F as ids / dists [n][degree] (-1 / +inf past a row's |F|).
+void oracle_forward_lists(const float* data, int64_t n, int32_t dim, int32_t metric,
+                          int32_t degree, int32_t* ids_out, float* dists_out, int32_t nthreads) {
+  auto F = forward_lists(data, n, dim, metric, degree, nthreads);
+  for (int64_t i = 0; i < n; ++i)
+    for (int j = 0; j < degree; ++j) {
+      const bool ok = j < (int)F[i].size();
+      ids_out[i * degree + j] = ok ? F[i][j].id : -1;
+      dists_out[i * degree + j] = ok ? F[i][j].dist : INFINITY;
+    }
+}
+
+// R16 steps on given forward lists: fwd_ids / fwd_dists [n][degree] (-1 /
+// any padding past a row's entries); the rows' keys are taken as given.
+void oracle_build_graph_from_forward(const float* data, int64_t n, int32_t dim, int32_t metric,
+                                     int32_t degree, const int32_t* fwd_ids,
+                                     const float* fwd_dists, int32_t* adj_out, int32_t nthreads) {
+  std::vector<std::vector<Key>> F(n);
+  for (int64_t i = 0; i < n; ++i)
+    for (int j = 0; j < degree; ++j) {
+      const int32_t id = fwd_ids[i * degree + j];
+      if (id >= 0) F[i].push_back(Key{fwd_dists[i * degree + j], id});
+    }
+  build_from_forward(data, n, dim, metric, degree, F, adj_out, nthreads);
 }
 
 // Cuckoo filter probe for tests of R10: applies ops[i] (+id = insert,

@@ -18,7 +18,7 @@ namespace {
 using song::fail;
 
 struct Scratch {
-  void* p[10] = {};
+  void* p[24] = {};
   int k = 0;
   ~Scratch() {
     for (int i = 0; i < k; ++i) cudaFree(p[i]);
@@ -83,50 +83,64 @@ int make_xmap(CUtensorMap* map, const float* x, int64_t n, int dim) {
                   "song_build_graph: %s: %s", #expr, cudaGetErrorString(e_));         \
   } while (0)
 
-extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, song_metric metric,
-                                int32_t degree, int32_t* adjacency_out, void* stream) {
-  using namespace song::graph;
-  if (!vectors || !adjacency_out) return fail(SONG_EINVAL, "NULL argument");
-  if (n < 1 || dim < 1 || degree < 1) return fail(SONG_EINVAL, "n, dim and degree must be >= 1");
-  if (n > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n must fit int32 ids");
-  if (degree > SONG_MAX_DEGREE)
-    return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
-  if (metric < SONG_L2 || metric > SONG_COSINE)
-    return fail(SONG_EINVAL, "metric %d: the builder takes SONG_L2, SONG_IP or SONG_COSINE",
-                (int)metric);
-  cudaStream_t st = (cudaStream_t)stream;
-  const int D = degree;
-  const int64_t nedges = n * (int64_t)D;
-  Scratch s;
-  float* norms = nullptr;
-  float* xs = nullptr;
-  uint64_t *fkeys = nullptr, *bkeys = nullptr, *inc = nullptr;
+namespace {
+using song::fail;
+
+// graph of rows [0, n) from the forward lists fkeys[0, n): R15 steps 2-4
+struct Finish {
+  uint64_t *bkeys = nullptr, *inc = nullptr;
   unsigned long long* cnt = nullptr;
   int64_t* off = nullptr;
   int *cursor = nullptr, *cnt32 = nullptr;
-  G_TRY(s.get(&norms, (n + 256) * sizeof(float)));  // (+ tail: tile-wide norm loads)
-  G_TRY(cudaMemsetAsync(norms, 0, (n + 256) * sizeof(float), st));
-  const float* x = vectors;
-  if (metric == SONG_COSINE) {  // normalise a scratch copy (1 - cos)
-    G_TRY(s.get(&xs, (size_t)n * dim * sizeof(float)));
-    G_TRY(cudaMemcpyAsync(xs, vectors, (size_t)n * dim * sizeof(float), cudaMemcpyDeviceToDevice, st));
-    x = xs;
+  void* tmp = nullptr;
+  size_t tmp_bytes = 0;
+  cudaError_t alloc(Scratch& s, int64_t n, int D, cudaStream_t st) {
+    const int64_t nedges = n * (int64_t)D;
+    cudaError_t e;
+    if ((e = s.get(&bkeys, nedges * sizeof(uint64_t)))) return e;
+    if ((e = s.get(&inc, nedges * sizeof(uint64_t)))) return e;
+    if ((e = s.get(&cnt, n * sizeof(unsigned long long)))) return e;
+    if ((e = s.get(&off, (n + 1) * sizeof(int64_t)))) return e;
+    if ((e = s.get(&cursor, n * sizeof(int)))) return e;
+    if ((e = s.get(&cnt32, n * sizeof(int)))) return e;
+    if ((e = cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, off, off, n, st))) return e;
+    return s.get(&tmp, tmp_bytes);
   }
-  G_TRY(s.get(&fkeys, nedges * sizeof(uint64_t)));
-  G_TRY(s.get(&bkeys, nedges * sizeof(uint64_t)));
-  G_TRY(s.get(&inc, nedges * sizeof(uint64_t)));
-  G_TRY(s.get(&cnt, n * sizeof(unsigned long long)));
-  G_TRY(s.get(&off, (n + 1) * sizeof(int64_t)));
-  G_TRY(s.get(&cursor, n * sizeof(int)));
-  G_TRY(s.get(&cnt32, n * sizeof(int)));
-  const int met = metric == SONG_L2 ? 0 : metric == SONG_IP ? 1 : 2;
-  const int blocks = (int)std::min<int64_t>((n + 7) / 8, 65535);
-  row_norms_kernel<<<blocks, 256, 0, st>>>(const_cast<float*>(x), n, dim, norms,
-                                           metric == SONG_COSINE);
+};
+
+int finish_graph(const float* x, int64_t n, int dim, int met, int D, const float* norms,
+                 const uint64_t* fkeys, Finish& f, int32_t* adjacency_out, cudaStream_t st) {
+  using namespace song::graph;
+  const int64_t nedges = n * (int64_t)D;
+  // 2. backward lists
+  G_TRY(cudaMemsetAsync(f.cnt, 0, n * sizeof(unsigned long long), st));
+  G_TRY(cudaMemsetAsync(f.cursor, 0, n * sizeof(int), st));
+  const int eb = (int)std::min<int64_t>((nedges + 255) / 256, 148 * 32);
+  count_u64_kernel<<<eb, 256, 0, st>>>(fkeys, nedges, f.cnt);
   G_TRY(cudaGetLastError());
-  // 1. forward lists: tensor cores (tcgen05, tf32) when that is exact for the
-  // data (every value tf32-representable, rows 16 B aligned), else fp32 FFMA
-  bool use_tc = dim % 4 == 0 && metric != SONG_COSINE;
+  i64_from_u64_kernel<<<eb, 256, 0, st>>>(f.cnt, f.off, n);
+  narrow_kernel<<<eb, 256, 0, st>>>(f.cnt, f.cnt32, n);
+  G_TRY(cudaGetLastError());
+  size_t tb = f.tmp_bytes;
+  G_TRY(cub::DeviceScan::ExclusiveSum(f.tmp, tb, f.off, f.off, n, st));
+  reverse_scatter_kernel<<<eb, 256, 0, st>>>(fkeys, nedges, D, f.off, f.cursor, f.inc);
+  G_TRY(cudaGetLastError());
+  const int blocks = (int)std::min<int64_t>((n + 7) / 8, 65535);
+  reverse_select_kernel<<<blocks, 256, 0, st>>>(f.inc, f.off, f.cnt32, n, D, f.bkeys);
+  G_TRY(cudaGetLastError());
+  // 3. + 4. candidates and the heuristic
+  const int pb = (int)std::min<int64_t>(n, 148 * 16);
+  prune_kernel<<<pb, PT, 0, st>>>(x, n, dim, norms, met, D, fkeys, f.bkeys, adjacency_out);
+  G_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+// R15 step 1 on rows [0, n): tensor cores (tcgen05, tf32) when that is exact
+// for the data (every value tf32-representable, rows 16 B aligned), else FFMA
+int forward_exact(const float* x, int64_t n, int dim, int met, bool cosine, int D,
+                  const float* norms, uint64_t* fkeys, Scratch& s, cudaStream_t st) {
+  using namespace song::graph;
+  bool use_tc = dim % 4 == 0 && !cosine;
   const char* force = std::getenv("SONG_GRAPH_PATH");  // "simt" / "tc" (tests, A/B)
   if (use_tc && !(force && std::strcmp(force, "tc") == 0)) {
     int* d_flag = nullptr;
@@ -157,28 +171,147 @@ extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, so
     knn_prefix_kernel<<<(unsigned)nb, THREADS, 0, st>>>(x, n, dim, norms, met, D, fkeys);
     G_TRY(cudaGetLastError());
   }
-  // 2. backward lists
-  G_TRY(cudaMemsetAsync(cnt, 0, n * sizeof(unsigned long long), st));
-  G_TRY(cudaMemsetAsync(cursor, 0, n * sizeof(int), st));
-  const int eb = (int)std::min<int64_t>((nedges + 255) / 256, 148 * 32);
-  count_u64_kernel<<<eb, 256, 0, st>>>(fkeys, nedges, cnt);
+  return SONG_OK;
+}
+
+int check_build_args(const float* vectors, int64_t n, int32_t dim, song_metric metric,
+                     int32_t degree, int32_t* adjacency_out) {
+  if (!vectors || !adjacency_out) return fail(SONG_EINVAL, "NULL argument");
+  if (n < 1 || dim < 1 || degree < 1) return fail(SONG_EINVAL, "n, dim and degree must be >= 1");
+  if (n > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "n must fit int32 ids");
+  if (degree > SONG_MAX_DEGREE)
+    return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
+  if (metric < SONG_L2 || metric > SONG_COSINE)
+    return fail(SONG_EINVAL, "metric %d: the builder takes SONG_L2, SONG_IP or SONG_COSINE",
+                (int)metric);
+  return SONG_OK;
+}
+
+// row norms (and the normalised scratch copy for cosine: 1 - cos)
+int prepare_rows(const float* vectors, int64_t n, int dim, song_metric metric, Scratch& s,
+                 float** norms, const float** x, cudaStream_t st) {
+  using namespace song::graph;
+  G_TRY(s.get(norms, (n + 256) * sizeof(float)));  // (+ tail: tile-wide norm loads)
+  G_TRY(cudaMemsetAsync(*norms, 0, (n + 256) * sizeof(float), st));
+  *x = vectors;
+  if (metric == SONG_COSINE) {
+    float* xs = nullptr;
+    G_TRY(s.get(&xs, (size_t)n * dim * sizeof(float)));
+    G_TRY(cudaMemcpyAsync(xs, vectors, (size_t)n * dim * sizeof(float), cudaMemcpyDeviceToDevice, st));
+    *x = xs;
+  }
+  const int blocks = (int)std::min<int64_t>((n + 7) / 8, 65535);
+  row_norms_kernel<<<blocks, 256, 0, st>>>(const_cast<float*>(*x), n, dim, *norms,
+                                           metric == SONG_COSINE);
   G_TRY(cudaGetLastError());
-  i64_from_u64_kernel<<<eb, 256, 0, st>>>(cnt, off, n);
-  narrow_kernel<<<eb, 256, 0, st>>>(cnt, cnt32, n);
-  G_TRY(cudaGetLastError());
-  size_t tmp_bytes = 0;
-  G_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, off, off, n, st));
-  void* tmp = nullptr;
-  G_TRY(s.get(&tmp, tmp_bytes));
-  G_TRY(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, off, off, n, st));
-  reverse_scatter_kernel<<<eb, 256, 0, st>>>(fkeys, nedges, D, off, cursor, inc);
-  G_TRY(cudaGetLastError());
-  reverse_select_kernel<<<blocks, 256, 0, st>>>(inc, off, cnt32, n, D, bkeys);
-  G_TRY(cudaGetLastError());
-  // 3. + 4. candidates and the heuristic
-  const int pb = (int)std::min<int64_t>(n, 148 * 16);
-  prune_kernel<<<pb, PT, 0, st>>>(x, n, dim, norms, met, D, fkeys, bkeys, adjacency_out);
-  G_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+// search results [nq][D] (ids, dists) -> forward keys (reading R16 step 2)
+__global__ void keys_from_results_kernel(const int32_t* __restrict__ ids,
+                                         const float* __restrict__ dists, int64_t cnt,
+                                         uint64_t* __restrict__ fkeys) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < cnt;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int id = ids[e];
+    fkeys[e] = id >= 0 ? song::make_key(dists[e], id) : song::KEY_MAX;
+  }
+}
+
+}  // namespace
+
+extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, song_metric metric,
+                                int32_t degree, int32_t* adjacency_out, void* stream) {
+  int rc = check_build_args(vectors, n, dim, metric, degree, adjacency_out);
+  if (rc) return rc;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int D = degree;
+  const int met = metric == SONG_L2 ? 0 : metric == SONG_IP ? 1 : 2;
+  Scratch s;
+  float* norms = nullptr;
+  const float* x = nullptr;
+  uint64_t* fkeys = nullptr;
+  if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
+  G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
+  // 1. forward lists
+  if ((rc = forward_exact(x, n, dim, met, metric == SONG_COSINE, D, norms, fkeys, s, st))) return rc;
+  // 2. - 4.
+  Finish f;
+  G_TRY(f.alloc(s, n, D, st));
+  if ((rc = finish_graph(x, n, dim, met, D, norms, fkeys, f, adjacency_out, st))) return rc;
   G_TRY(cudaStreamSynchronize(st));  // the scratch is freed on return
+  return SONG_OK;
+}
+
+extern "C" int song_build_graph_batched(const float* vectors, int64_t n, int32_t dim,
+                                        song_metric metric, int32_t degree, int32_t prefix,
+                                        int32_t queue_len, int32_t batch_shift,
+                                        int32_t* adjacency_out, void* stream) {
+  int rc = check_build_args(vectors, n, dim, metric, degree, adjacency_out);
+  if (rc) return rc;
+  if (prefix < 1) return fail(SONG_EINVAL, "prefix %d < 1", prefix);
+  if (queue_len < degree || queue_len > SONG_MAX_QUEUE_LEN)
+    return fail(SONG_EINVAL, "queue_len %d outside [degree, %d]", queue_len, SONG_MAX_QUEUE_LEN);
+  if (batch_shift < 0 || batch_shift > 16) return fail(SONG_EINVAL, "batch_shift %d outside [0, 16]", batch_shift);
+  cudaStream_t st = (cudaStream_t)stream;
+  const int D = degree;
+  const int met = metric == SONG_L2 ? 0 : metric == SONG_IP ? 1 : 2;
+  Scratch s;
+  float* norms = nullptr;
+  const float* x = nullptr;
+  uint64_t* fkeys = nullptr;
+  if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
+  G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
+  // 1. exact forward lists of the prefix (R15 step 1)
+  const int64_t m0 = std::min<int64_t>(n, prefix);
+  if ((rc = forward_exact(x, m0, dim, met, metric == SONG_COSINE, D, norms, fkeys, s, st))) return rc;
+  Finish f;
+  G_TRY(f.alloc(s, n, D, st));
+  if (m0 < n) {
+    // the search's view of the rows: [n][dpad] (16 B rows; normalised for cosine)
+    const int dpad = (dim + 3) & ~3;
+    const float* xv = x;
+    if (dpad != dim) {
+      float* xp = nullptr;
+      G_TRY(s.get(&xp, (size_t)n * dpad * sizeof(float)));
+      G_TRY(cudaMemsetAsync(xp, 0, (size_t)n * dpad * sizeof(float), st));
+      G_TRY(cudaMemcpy2DAsync(xp, dpad * sizeof(float), x, dim * sizeof(float), dim * sizeof(float),
+                              n, cudaMemcpyDeviceToDevice, st));
+      xv = xp;
+    }
+    const int64_t CH = 1 << 22;  // queries per search launch
+    int32_t* ids = nullptr;
+    float* dists = nullptr;
+    G_TRY(s.get(&ids, CH * D * sizeof(int32_t)));
+    G_TRY(s.get(&dists, CH * D * sizeof(float)));
+    song_search_params p;
+    song_default_params(&p, D, queue_len);
+    song_index* view = nullptr;
+    if ((rc = song::make_search_view(xv, n, dim, D, (int)metric, adjacency_out, &view))) return rc;
+    int64_t m = m0;
+    while (m < n && rc == SONG_OK) {
+      const int64_t b = std::min<int64_t>(n - m, std::max<int64_t>(1, m >> batch_shift));
+      // G_m = R15 steps 2-4 on F of rows [0, m), into adjacency rows [0, m)
+      if ((rc = finish_graph(x, m, dim, met, D, norms, fkeys, f, adjacency_out, st))) break;
+      // every row of the batch searches G_m: F(i) = its top D (ids < m)
+      for (int64_t c0 = m; c0 < m + b && rc == SONG_OK; c0 += CH) {
+        const int64_t nc = std::min<int64_t>(CH, m + b - c0);
+        rc = song::search_view(view, m, &p, vectors + c0 * dim, nc, ids, dists, st);
+        if (rc) break;
+        const int kb = (int)std::min<int64_t>((nc * D + 255) / 256, 148 * 32);
+        keys_from_results_kernel<<<kb, 256, 0, st>>>(ids, dists, nc * D, fkeys + c0 * D);
+        if (cudaGetLastError() != cudaSuccess) rc = fail(SONG_ECUDA, "keys_from_results launch");
+      }
+      m += b;
+    }
+    int status = 0;
+    if (rc == SONG_OK) rc = song::view_status(view, &status, st);
+    song::free_search_view(view);
+    if (rc) return rc;
+    if (status & song::STATUS_BAD_INPUT) return fail(SONG_EINVAL, "vectors hold non-finite values");
+  }
+  // 3. the graph on all rows
+  if ((rc = finish_graph(x, n, dim, met, D, norms, fkeys, f, adjacency_out, st))) return rc;
+  G_TRY(cudaStreamSynchronize(st));
   return SONG_OK;
 }

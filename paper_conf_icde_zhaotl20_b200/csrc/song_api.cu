@@ -473,6 +473,59 @@ int alloc_codes_index(int64_t n, int32_t bits, const int32_t* adjacency, int32_t
 
 }  // namespace
 
+namespace song {
+int make_search_view(const float* xv, int64_t n, int dim, int degree, int metric, int32_t* adj,
+                     song_index** out) {
+  song_index* ix = new song_index();
+  cudaError_t e = cudaGetDevice(&ix->device);
+  if (e == cudaSuccess)
+    e = cudaDeviceGetAttribute(&ix->num_sms, cudaDevAttrMultiProcessorCount, ix->device);
+  if (e == cudaSuccess) e = cudaMalloc(&ix->d_ticket, sizeof(unsigned));
+  if (e == cudaSuccess) e = cudaMalloc(&ix->d_status, sizeof(int));
+  if (e == cudaSuccess) e = cudaMemset(ix->d_status, 0, sizeof(int));
+  ix->n = n;
+  ix->dim = dim;
+  ix->dpad = (dim + 3) & ~3;
+  ix->degree = degree;
+  ix->metric = metric;
+  ix->d_data = const_cast<float*>(xv);
+  ix->d_adj = adj;
+  ix->dedup = 1;
+  if (e != cudaSuccess) {
+    free_search_view(ix);
+    return fail(e == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA, "search view: %s",
+                cudaGetErrorString(e));
+  }
+  *out = ix;
+  return SONG_OK;
+}
+
+int search_view(song_index* view, int64_t m, const song_search_params* p, const float* q,
+                int64_t nq, int32_t* ids, float* dists, cudaStream_t st) {
+  view->n = m;
+  return enqueue_search(view, p, q, nq, ids, dists, nullptr, st);
+}
+
+int view_status(song_index* view, int* status, cudaStream_t st) {
+  CUDA_TRY(cudaMemcpyAsync(status, view->d_status, sizeof(int), cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  return SONG_OK;
+}
+
+void free_search_view(song_index* view) {
+  if (!view) return;
+  view->d_data = nullptr;  // not owned
+  view->d_adj = nullptr;
+  cudaFree(view->d_ticket);
+  cudaFree(view->d_status);
+  cudaFree(view->d_gtab);
+  cudaFree(view->d_order);
+  cudaFree(view->d_qbin);
+  cudaFree(view->d_bins);
+  delete view;
+}
+}  // namespace song
+
 extern "C" {
 
 int song_rp_encode(const float* vectors, int64_t n, int32_t dim, const float* R, int32_t bits,

@@ -46,6 +46,16 @@ struct song_index {
 
 namespace song {
 int fail(int code, const char* fmt, ...);
+// non-owning search index over device rows (the batched graph builder, R16):
+// xv [n][dpad] rows (normalised for cosine), adj [n][degree]; the view never
+// frees them
+int make_search_view(const float* xv, int64_t n, int dim, int degree, int metric, int32_t* adj,
+                     song_index** out);
+// search the view restricted to its first m rows (entry 0; ids < m)
+int search_view(song_index* view, int64_t m, const song_search_params* p, const float* q,
+                int64_t nq, int32_t* ids, float* dists, cudaStream_t st);
+int view_status(song_index* view, int* status, cudaStream_t st);
+void free_search_view(song_index* view);
 }  // namespace song
 
 #define CUDA_TRY(expr)                                                                  \

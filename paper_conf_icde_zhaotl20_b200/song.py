@@ -33,7 +33,7 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
-            "song_search_codes_ex", "song_build_graph"]
+            "song_search_codes_ex", "song_build_graph", "song_build_graph_batched"]
 
 
 class SongError(RuntimeError):
@@ -91,6 +91,7 @@ def lib():
         L.song_index_create_rp.argtypes = [P, i64, i32, P, i32, P, i32, PP]
         L.song_search_codes_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
         L.song_build_graph.argtypes = [P, i64, i32, i32, i32, P, P]
+        L.song_build_graph_batched.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, P, P]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -99,7 +100,7 @@ def lib():
                      "song_index_get_info", "song_search", "song_search_ex",
                      "song_index_last_status", "song_merge_topk", "song_rp_encode",
                      "song_index_create_codes", "song_index_create_rp",
-                     "song_search_codes_ex", "song_build_graph"):
+                     "song_search_codes_ex", "song_build_graph", "song_build_graph_batched"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -336,6 +337,25 @@ def build_graph(vectors, degree: int = 32, metric: str = "l2"):
         _check(lib().song_build_graph(ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1],
                                       METRICS[metric], degree, ctypes.c_void_p(adj.data_ptr()),
                                       _stream_ptr(v.device)))
+    return adj
+
+
+def build_graph_batched(vectors, degree: int = 32, metric: str = "l2", prefix: int = 1 << 20,
+                        queue_len: int = 64, batch_shift: int = 1):
+    """song_build_graph_batched (reading R16, the scale-out builder):
+    exact forward lists for the first `prefix` rows, then batches of
+    max(1, m >> batch_shift) rows search the graph of the rows before them
+    (K = degree, `queue_len`) for their forward lists."""
+    torch = _torch()
+    if not _is_cuda_tensor(vectors):
+        raise TypeError("build_graph_batched() takes a CUDA tensor")
+    v = vectors.contiguous().float()
+    adj = torch.empty((v.shape[0], degree), dtype=torch.int32, device=v.device)
+    with torch.cuda.device(v.device):
+        _check(lib().song_build_graph_batched(
+            ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1], METRICS[metric], degree,
+            int(prefix), int(queue_len), int(batch_shift), ctypes.c_void_p(adj.data_ptr()),
+            _stream_ptr(v.device)))
     return adj
 
 

@@ -99,3 +99,64 @@ def test_errors():
         with pytest.raises(s.SongError) as e:
             s.build_graph(x, D)
         assert e.value.code == code
+
+
+# ------------------------------------------- batched insertion (reading R16)
+def gbuild_batched(x, D, metric="l2", **kw):
+    adj = song().build_graph_batched(torch.as_tensor(x, device="cuda"), D, metric, **kw)
+    torch.cuda.synchronize()
+    return adj.cpu().numpy()
+
+
+@pytest.mark.parametrize("n,dim,D,prefix,L,shift", [
+    (600, 8, 6, 100, 600, 1),      # exhaustive searches (the pinned special case)
+    (3000, 30, 12, 200, 32, 1),    # dim % 4 != 0: the padded search view
+    (5000, 16, 16, 500, 48, 0),    # doubling batches
+    (4097, 64, 32, 1000, 64, 2),   # ragged last batch
+])
+def test_batched_integer_bit_exact(n, dim, D, prefix, L, shift):
+    x = og._int_data(n, dim, n)
+    want = oracle.build_graph_batched(x, D, prefix=prefix, queue_len=L, batch_shift=shift,
+                                      nthreads=8)
+    np.testing.assert_array_equal(gbuild_batched(x, D, prefix=prefix, queue_len=L,
+                                                 batch_shift=shift), want)
+
+
+def test_batched_sift_shaped_bit_exact():
+    cfg = CONFIGS["sift1m"]
+    x, _ = make_data(cfg, device="cuda", n=20_000, nq=1)
+    got = gbuild_batched(x, 32, prefix=2000, queue_len=64, batch_shift=1)
+    want = oracle.build_graph_batched(x.cpu().numpy(), 32, prefix=2000, queue_len=64,
+                                      batch_shift=1, nthreads=16)
+    np.testing.assert_array_equal(got, want)
+
+
+def test_batched_whole_prefix_is_song_build_graph():
+    x = og._int_data(3000, 32, 11)
+    np.testing.assert_array_equal(gbuild_batched(x, 16, prefix=3000), gbuild(x, 16))
+
+
+@pytest.mark.parametrize("metric", ["ip", "cosine"])
+def test_batched_float_metrics_search_well(metric):
+    cfg = CONFIGS["glove200" if metric == "ip" else "nytimes256"]
+    x, q = make_data(cfg, device="cuda", n=20_000, nq=200)
+    s = song()
+    adj = s.build_graph_batched(x, 32, metric, prefix=2000, queue_len=64)
+    exact = s.build_graph(x, 32, metric)
+    truth = oracle.bruteforce(x.cpu().numpy(), q.cpu().numpy(), 10,
+                              metric=oracle.METRICS[metric])[0]
+    rec = []
+    for g in (adj, exact):
+        idx = s.SongIndex(x, g, metric=metric)
+        ids, _ = idx.search(q, params=s.Params(K=10, queue_len=256))
+        rec.append(oracle.recall(ids.cpu().numpy(), truth))
+        idx.close()
+    assert rec[0] >= rec[1] - 0.05, rec
+
+
+def test_batched_errors():
+    s = song()
+    x = torch.zeros((100, 8), device="cuda")
+    for kw in (dict(prefix=0), dict(queue_len=4), dict(batch_shift=17)):
+        with pytest.raises(s.SongError):
+            s.build_graph_batched(x, 8, **kw)

@@ -95,3 +95,75 @@ def test_agrees_with_the_torch_tooling():
     same_rows = (a == b).all(1).mean()
     same_sets = np.mean([set(r) == set(s) for r, s in zip(a, b)])
     assert same_sets >= 0.99 and same_rows >= 0.98
+
+
+# ---------------------------------------------------------------- reading R16
+def _int_data(n, dim, seed):
+    rng = np.random.default_rng(seed)
+    return rng.integers(0, 64, size=(n, dim)).astype(np.float32)
+
+
+def test_forward_lists_match_bruteforce():
+    x = _int_data(300, 8, 3)
+    ids, dists = oracle.forward_lists(x, 6)
+    for i, keys in enumerate(_forward_bruteforce(x, 6)[1]):
+        assert [int(j) for j in ids[i] if j >= 0] == [j for _, j in keys]
+        np.testing.assert_array_equal(dists[i, :len(keys)], [d for d, _ in keys])
+
+
+def test_batched_with_whole_prefix_is_r15():
+    """prefix >= n: no batches, R16 reduces to R15."""
+    x = _int_data(400, 8, 4)
+    np.testing.assert_array_equal(oracle.build_graph_batched(x, 8, prefix=400),
+                                  oracle.build_graph(x, 8))
+
+
+def test_batch_bounds():
+    assert oracle.batch_bounds(10, 4, 1) == [(4, 6), (6, 9), (9, 10)]
+    assert oracle.batch_bounds(10, 4, 0) == [(4, 8), (8, 10)]
+    assert oracle.batch_bounds(3, 5, 1) == []
+
+
+def test_batched_full_queue_equals_batch_restricted_definition():
+    """With queue_len >= the searched prefix every search is exhaustive, so F(i)
+    is the D nearest rows among those reachable from entry 0 in G_m (m = start
+    of i's batch) — computed here by BFS + numpy brute force, independent of
+    the oracle's search — and the graph is R15 steps 2-4 on those lists."""
+    n, D, prefix, shift = 600, 6, 100, 1
+    x = _int_data(n, 8, 5)
+    d = ((x[:, None, :].astype(np.float64) - x[None, :, :]) ** 2).sum(-1).astype(np.float32)
+    fi = np.full((n, D), -1, np.int32)
+    fd = np.full((n, D), np.inf, np.float32)
+    for i, keys in enumerate(_forward_bruteforce(x[:prefix], D)[1]):
+        for t, (dd, j) in enumerate(keys):
+            fi[i, t], fd[i, t] = j, dd
+    for m, m1 in oracle.batch_bounds(n, prefix, shift):
+        g = oracle.build_graph_from_forward(x[:m], fi[:m], fd[:m])
+        seen, stack = {0}, [0]
+        while stack:
+            for u in g[stack.pop()]:
+                if u >= 0 and int(u) not in seen:
+                    seen.add(int(u))
+                    stack.append(int(u))
+        for i in range(m, m1):
+            keys = sorted((d[i, j], j) for j in seen)[:D]
+            for t, (dd, j) in enumerate(keys):
+                fi[i, t], fd[i, t] = j, dd
+    want = oracle.build_graph_from_forward(x, fi, fd)
+    got = oracle.build_graph_batched(x, D, prefix=prefix, queue_len=n, batch_shift=shift)
+    np.testing.assert_array_equal(got, want)
+
+
+def test_batched_graph_is_valid_and_searchable():
+    x = _int_data(2000, 16, 6)
+    D = 8
+    adj = oracle.build_graph_batched(x, D, prefix=200, queue_len=32, batch_shift=1)
+    assert adj.shape == (2000, D)
+    assert ((adj >= -1) & (adj < 2000)).all()
+    for v, row in enumerate(adj):
+        r = [int(j) for j in row if j >= 0]
+        assert v not in r and len(set(r)) == len(r)
+    q = _int_data(50, 16, 7)
+    ids, _, _, _ = oracle.search(x, adj, q, 10, 64)
+    truth, _ = oracle.bruteforce(x, q, 10)
+    assert oracle.recall(ids, truth) > 0.9

@@ -1,0 +1,139 @@
+"""Scale-out config (BASELINE.json configs[4]) on one B200: the SIFT-shaped
+generator at n rows (default 100M), the graph built by song_build_graph_batched
+(reading R16: the exact R15 builder is O(n^2)), then QPS at
+recall@10 >= 0.95 over 10,000 fresh queries (query-sharded mode: every GPU of
+the scale-out holds this replica and searches its own batch).  With
+--compare-exact (n <= a few million) the R15 graph is built too and both
+recall curves are reported.
+
+    python tools/bench_scaleout.py [--n 100000000] [--out gpurun_out/scaleout.json]
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+GRID = [10, 12, 16, 20, 24, 32, 40, 48, 64, 80, 96, 128, 160, 192, 256]
+
+
+def exact_topk(x, q, K, qchunk=1024, xchunk=1 << 21):
+    """Brute-force top-K (squared L2, fp32 GEMM, TF32 off; exact on the integer
+    data) over x in chunks, merged by (dist, id)."""
+    import torch
+    torch.backends.cuda.matmul.allow_tf32 = False
+    out = []
+    for s in range(0, q.shape[0], qchunk):
+        qq = q[s:s + qchunk]
+        qn = (qq * qq).sum(1, keepdim=True)
+        best_d = torch.full((qq.shape[0], K), float("inf"), device=q.device)
+        best_i = torch.full((qq.shape[0], K), -1, dtype=torch.int64, device=q.device)
+        for c in range(0, x.shape[0], xchunk):
+            xc = x[c:c + xchunk]
+            d = qn + (xc * xc).sum(1)[None] - 2 * qq @ xc.T
+            v, i = torch.topk(d, K, dim=1, largest=False)
+            cd = torch.cat([best_d, v], 1)
+            ci = torch.cat([best_i, i + c], 1)
+            # (dist, id) order: ids break ties
+            key = cd.double() * 4e9 + ci.double()
+            o = torch.argsort(key, dim=1)[:, :K]
+            best_d, best_i = torch.gather(cd, 1, o), torch.gather(ci, 1, o)
+            del d
+        out.append(best_i)
+    return torch.cat(out).int()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=100_000_000)
+    ap.add_argument("--nq", type=int, default=10_000)
+    ap.add_argument("--prefix", type=int, default=1 << 20)
+    ap.add_argument("--build-queue-len", type=int, default=64)
+    ap.add_argument("--batch-shift", type=int, default=1)
+    ap.add_argument("--compare-exact", action="store_true")
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--out", default="gpurun_out/scaleout.json")
+    a = ap.parse_args()
+    import numpy as np
+    import torch
+    import bench
+    from paper_conf_icde_zhaotl20_b200 import song
+    from workloads.synth import CONFIGS, generator_for
+    cfg = CONFIGS["scaleout100m"]
+    dev = torch.device("cuda", 0)
+    t0 = time.time()
+    gen = generator_for(cfg, dev)
+    x = gen.sample(a.n, cfg.seed)
+    q = gen.sample(a.nq, cfg.seed + 1)
+    torch.cuda.synchronize()
+    res = {"n": a.n, "nq": a.nq, "dim": 128, "degree": 32, "data_s": round(time.time() - t0, 1),
+           "builder": {"prefix": a.prefix, "queue_len": a.build_queue_len,
+                       "batch_shift": a.batch_shift}}
+    print(res, flush=True)
+    t0 = time.time()
+    truth = exact_topk(x, q, 10).cpu().numpy()
+    torch.cuda.synchronize()
+    res["truth_s"] = round(time.time() - t0, 1)
+    graphs = {}
+    t0 = time.time()
+    graphs["batched"] = song.build_graph_batched(x, 32, "l2", prefix=a.prefix,
+                                                 queue_len=a.build_queue_len,
+                                                 batch_shift=a.batch_shift)
+    torch.cuda.synchronize()
+    res["build_s"] = round(time.time() - t0, 1)
+    print("built", res["build_s"], "s", flush=True)
+    if a.compare_exact:
+        t0 = time.time()
+        graphs["exact"] = song.build_graph(x, 32, "l2")
+        torch.cuda.synchronize()
+        res["build_exact_s"] = round(time.time() - t0, 1)
+    for name, adj in graphs.items():
+        idx = song.SongIndex(x, adj)
+        del adj
+        sweep, L_op = [], None
+        for L in GRID:
+            ids, _ = idx.search(q, params=song.Params(K=10, queue_len=L))
+            r = bench.recall_t(ids, torch.as_tensor(truth, device=dev))
+            sweep.append((L, round(r, 4)))
+            if r >= 0.95 and L_op is None:
+                L_op = L
+                break
+        row = {"recall_sweep": sweep, "queue_len": L_op}
+        if L_op:
+            p = song.Params(K=10, queue_len=L_op)
+            out = (torch.empty((a.nq, 10), dtype=torch.int32, device=dev),
+                   torch.empty((a.nq, 10), dtype=torch.float32, device=dev), None)
+            _, _, ctr = idx.search(q, params=p, counters=True)
+            flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+            for _ in range(3):
+                idx.search(q, params=p, out=out)
+            ts = []
+            for _ in range(a.steps):
+                flush.zero_()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                idx.search(q, params=p, out=out)
+                e1.record()
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ms = float(np.mean(ts))
+            n_dist, n_exp = int(ctr[:, 0].long().sum()), int(ctr[:, 1].long().sum())
+            alg = 512 * n_dist + 128 * n_exp + 512 * a.nq + 80 * a.nq
+            peak, _ = bench.measured_peak_hbm()
+            row.update({"qps": round(a.nq / ms * 1e3, 1), "ms_per_step": round(ms, 4),
+                        "n_dist": n_dist, "n_exp": n_exp,
+                        "roofline_frac": round(alg / (ms / 1e3) / 1e9 / peak, 4)})
+        idx.close()
+        res[name] = row
+        print(name, row, flush=True)
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    with open(a.out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    main()

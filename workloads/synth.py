@@ -39,6 +39,9 @@ CONFIGS = {
     "nytimes256": Config("nytimes256", 289_761, 256, "cosine", 32, 10_000, 10, 400, "nytimes"),
     # §VII / Fig. 14: MNIST8m and its 1M sample, searched top-1 through
     # 1-bit random-projection codes of h bits (extra["hash_bits"])
+    # BASELINE.json configs[4] (scale-out): the SIFT1M generator at 100M rows
+    # (51.2 GB + a 12.8 GB graph: one B200 holds a replica); s = 500
+    "scaleout100m": Config("scaleout100m", 100_000_000, 128, "l2", 32, 10_000, 10, 500, "sift"),
     "mnist1m": Config("mnist1m", 1_000_000, 784, "l2", 32, 10_000, 1, 600, "mnist",
                       extra={"hash_bits": 128}),
     "mnist8m": Config("mnist8m", 8_090_000, 784, "l2", 32, 10_000, 1, 600, "mnist",
