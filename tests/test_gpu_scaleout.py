@@ -1,0 +1,54 @@
+"""BASELINE.json configs[4] (scale-out) at full size on one B200: 100M x 128
+SIFT-shaped rows (51.2 GB) and their degree-32 graph (12.8 GB) built on the
+device by song_build_graph_batched (reading R16; the exact R15 builder is
+O(n^2)), one replica searched with the 10,000-query batch at queue_len 64 (the
+recall@10 >= 0.95 operating point of tools/bench_scaleout.py,
+profiles/r01m_scaleout_100m.json).  The oracle recomputes 100 sampled queries
+one by one: ids, distances and counters bit-exact (integer data, pin P8).
+
+Skipped when the GPU or the host cannot hold the config (~150 GB of device
+memory while the graph is built, ~70 GB of host memory for the oracle)."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+import oracle  # noqa: E402
+from workloads.synth import CONFIGS, generator_for  # noqa: E402
+
+from test_gpu_parity import assert_exact, oracle_kw, song  # noqa: E402
+
+
+def test_scaleout_100m_sampled_parity():
+    import psutil
+    s = song()
+    torch.cuda.empty_cache()
+    free, _ = torch.cuda.mem_get_info()
+    if free < 150 * 2**30 or psutil.virtual_memory().available < 90 * 2**30:
+        pytest.skip(f"needs ~150 GB GPU / 90 GB host memory (free GPU {free / 2**30:.0f} GB)")
+    cfg = CONFIGS["scaleout100m"]
+    gen = generator_for(cfg, "cuda")
+    x = gen.sample(cfg.n, cfg.seed)
+    q = gen.sample(cfg.nq, cfg.seed + 1)
+    adj = s.build_graph_batched(x, cfg.degree, cfg.metric, prefix=1 << 16, queue_len=64,
+                                batch_shift=1)
+    torch.cuda.synchronize()
+    idx = s.SongIndex(x, adj)
+    ids, d, c = idx.search(q, params=s.Params(K=cfg.K, queue_len=64), counters=True)
+    torch.cuda.synchronize()
+    idx.last_status()
+    idx.close()
+    pick = np.arange(0, cfg.nq, cfg.nq // 100)
+    gi, gd, gc = ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy()
+    an = adj.cpu().numpy()
+    del adj
+    xn = x.cpu().numpy()
+    o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 64, nthreads=16,
+                      **oracle_kw("hash", 64))
+    assert_exact((gi[pick], gd[pick], gc[pick]), o)
+    # every row of the graph: ids in range, no self loop, no repeats (sampled rows)
+    rows = an[np.random.default_rng(0).choice(cfg.n, 20_000, replace=False)]
+    assert ((rows >= -1) & (rows < cfg.n)).all()
+    assert all(len(set(r[r >= 0])) == (r >= 0).sum() for r in rows)
+    assert (np.diff(gd, axis=1) >= 0).all()

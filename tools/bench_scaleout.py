@@ -50,11 +50,13 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=100_000_000)
     ap.add_argument("--nq", type=int, default=10_000)
-    ap.add_argument("--prefix", type=int, default=1 << 20)
+    ap.add_argument("--prefix", type=int, default=1 << 16)
     ap.add_argument("--build-queue-len", type=int, default=64)
     ap.add_argument("--batch-shift", type=int, default=1)
     ap.add_argument("--compare-exact", action="store_true")
     ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--parity-sample", type=int, default=0,
+                    help="queries the oracle recomputes one by one at the operating point")
     ap.add_argument("--out", default="gpurun_out/scaleout.json")
     a = ap.parse_args()
     import numpy as np
@@ -69,7 +71,13 @@ def main():
     x = gen.sample(a.n, cfg.seed)
     q = gen.sample(a.nq, cfg.seed + 1)
     torch.cuda.synchronize()
-    res = {"n": a.n, "nq": a.nq, "dim": 128, "degree": 32, "data_s": round(time.time() - t0, 1),
+    import psutil
+    need = a.n * (128 * 4 + 32 * 4) * 1.6
+    if a.parity_sample and psutil.virtual_memory().available < need:
+        print(f"parity sample skipped: {psutil.virtual_memory().available / 2**30:.0f} GB host RAM "
+              f"available, {need / 2**30:.0f} GB needed", flush=True)
+        a.parity_sample = 0
+    res = {"host_ram_gb": round(psutil.virtual_memory().total / 2**30, 1), "n": a.n, "nq": a.nq, "dim": 128, "degree": 32, "data_s": round(time.time() - t0, 1),
            "builder": {"prefix": a.prefix, "queue_len": a.build_queue_len,
                        "batch_shift": a.batch_shift}}
     print(res, flush=True)
@@ -77,6 +85,7 @@ def main():
     truth = exact_topk(x, q, 10).cpu().numpy()
     torch.cuda.synchronize()
     res["truth_s"] = round(time.time() - t0, 1)
+    torch.cuda.empty_cache()
     graphs = {}
     t0 = time.time()
     graphs["batched"] = song.build_graph_batched(x, 32, "l2", prefix=a.prefix,
@@ -92,7 +101,10 @@ def main():
         res["build_exact_s"] = round(time.time() - t0, 1)
     for name, adj in graphs.items():
         idx = song.SongIndex(x, adj)
+        adj_host = adj.cpu().numpy() if a.parity_sample else None
         del adj
+        graphs[name] = None
+        torch.cuda.empty_cache()
         sweep, L_op = [], None
         for L in GRID:
             ids, _ = idx.search(q, params=song.Params(K=10, queue_len=L))
@@ -120,6 +132,20 @@ def main():
                 torch.cuda.synchronize()
                 ts.append(e0.elapsed_time(e1))
             ms = float(np.mean(ts))
+            if a.parity_sample:
+                import oracle
+                pick = np.arange(0, a.nq, max(1, a.nq // a.parity_sample))[:a.parity_sample]
+                gi, gd, gc = (t.cpu().numpy() for t in idx.search(q, params=p, counters=True))
+                cap = int(__import__("paper_conf_icde_zhaotl20_b200.song", fromlist=["x"]).default_visited_cap(L_op))
+                t1 = time.time()
+                oi, od, oc, _ = oracle.search(x.cpu().numpy(), adj_host, q.cpu().numpy()[pick], 10,
+                                              L_op, flags=oracle.OPTIMIZED_LAZY, lazy_cap=cap,
+                                              nthreads=os.cpu_count() or 8)
+                row["parity_sample"] = {
+                    "queries": len(pick), "oracle_s": round(time.time() - t1, 1),
+                    "ids_equal": float((gi[pick] == oi).all(1).mean()),
+                    "dists_equal": float((gd[pick] == od).all(1).mean()),
+                    "counters_equal": float((gc[pick].astype(np.int64) == oc).all(1).mean())}
             n_dist, n_exp = int(ctr[:, 0].long().sum()), int(ctr[:, 1].long().sum())
             alg = 512 * n_dist + 128 * n_exp + 512 * a.nq + 80 * a.nq
             peak, _ = bench.measured_peak_hbm()
