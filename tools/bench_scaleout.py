@@ -46,6 +46,56 @@ def exact_topk(x, q, K, qchunk=1024, xchunk=1 << 21):
     return torch.cat(out).int()
 
 
+def sharded(a, x, q, truth, song, bench, torch, np):
+    """Dataset sharding on one GPU: shard g = rows [lo_g, hi_g) with its own
+    R16 graph; each shard searches the whole batch (id_offset = lo_g) — on a
+    G-GPU node the G searches run concurrently, so the step is the slowest
+    shard's search + the merge — and song_merge_topk keeps the K best."""
+    from paper_conf_icde_zhaotl20_b200.sharded import shard_ranges
+    G, dev = a.shards, q.device
+    idxs = []
+    t0 = time.time()
+    for lo, hi in shard_ranges(a.n, G):
+        adj = song.build_graph_batched(x[lo:hi], 32, "l2", prefix=a.prefix,
+                                       queue_len=a.build_queue_len, batch_shift=a.batch_shift)
+        idxs.append((lo, song.SongIndex(x[lo:hi], adj)))
+        del adj
+        torch.cuda.empty_cache()
+    build_s = time.time() - t0
+    out = {"shards": G, "build_s_total": round(build_s, 1), "sweep": []}
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    for L in GRID:
+        ids_g, d_g, shard_ms = [], [], []
+        for lo, idx in idxs:
+            p = song.Params(K=10, queue_len=L, id_offset=lo)
+            idx.search(q, params=p)
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            i, d = idx.search(q, params=p)
+            e1.record()
+            torch.cuda.synchronize()
+            shard_ms.append(e0.elapsed_time(e1))
+            ids_g.append(i)
+            d_g.append(d)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        mi, _ = song.merge_topk(torch.stack(ids_g), torch.stack(d_g), 10)
+        e1.record()
+        torch.cuda.synchronize()
+        r = bench.recall_t(mi, torch.as_tensor(truth, device=dev))
+        step_ms = max(shard_ms) + e0.elapsed_time(e1)
+        out["sweep"].append({"L": L, "recall": round(r, 4), "max_shard_ms": round(max(shard_ms), 4),
+                             "merge_ms": round(e0.elapsed_time(e1), 4),
+                             "qps_G_gpus": round(a.nq / step_ms * 1e3, 1)})
+        if r >= 0.95:
+            out["queue_len"] = L
+            break
+    for _, idx in idxs:
+        idx.close()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=100_000_000)
@@ -57,6 +107,10 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--parity-sample", type=int, default=0,
                     help="queries the oracle recomputes one by one at the operating point")
+    ap.add_argument("--shards", type=int, default=0,
+                    help="also run dataset sharding (P:471, SURVEY §8(e)(ii)): G shards with "
+                         "their own graphs, every query searched on every shard, merged by "
+                         "song_merge_topk; emulated on this GPU one shard at a time")
     ap.add_argument("--out", default="gpurun_out/scaleout.json")
     a = ap.parse_args()
     import numpy as np
@@ -155,6 +209,9 @@ def main():
         idx.close()
         res[name] = row
         print(name, row, flush=True)
+    if a.shards:
+        res["dataset_sharded"] = sharded(a, x, q, truth, song, bench, torch, np)
+        print("dataset_sharded", res["dataset_sharded"], flush=True)
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(res, f, indent=1)
