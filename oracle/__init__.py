@@ -6,11 +6,13 @@ paper.  Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
 product package ``paper_conf_icde_zhaotl20_b200`` never imports it and shares
 no code with it (the C++ source is ``oracle/song_oracle.cpp``; the readings
-R1-R15 it follows are listed in its header and in DESIGN.md §3).
+R1-R16 it follows are listed in its header and in DESIGN.md §3).
 
 This module only marshals numpy arrays into ``liboracle.so`` (built by
 :func:`build`) and adds the two plain definitions the paper states in prose:
-recall and the merge of per-shard results.
+recall and the merge of per-shard results, plus the batch
+loop of reading R16 (:func:`build_graph_batched`), which composes the C++
+forward lists, graph steps and search in the order the reading states.
 """
 from __future__ import annotations
 

@@ -62,6 +62,13 @@
 //         and d(c, k) > d(c, v) for every kept k ("closer to the base than to
 //         every kept neighbour"); then refill with the skipped candidates in
 //         C(v) order up to D; pad with -1.  Row = kept then refilled, in order.
+//   R16 batched-insertion construction (the scale-out builder; the batch loop
+//      is in oracle/__init__.py build_graph_batched): rows [0, P) take R15's
+//      forward lists; each later batch [m, m + max(1, m >> s)) searches the
+//      graph G_m = R15 steps 2-4 on the forward lists of rows [0, m)
+//      (Algorithm 1, entry 0, K = D) and takes the top D as forward lists;
+//      the graph is R15 steps 2-4 on all rows (oracle_forward_lists,
+//      oracle_build_graph_from_forward below).
 //   R12 Hamming search: the distance of two codes is the number of differing
 //      bits ("the hamming distance between the bit-vectors"), used as the
 //      key's distance (an integer, exact in fp32) with the same (dist, id)
