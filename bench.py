@@ -66,6 +66,9 @@ def parse():
     ap.add_argument("--graph", default="auto", choices=GRAPH_BUILDERS,
                     help="graph builder: batched insertion (R16) / exact insertion (R15) / "
                          "auto = per metric (default_graph)")
+    ap.add_argument("--build-prefix", type=int, default=0)
+    ap.add_argument("--build-queue-len", type=int, default=0)
+    ap.add_argument("--build-shift", type=int, default=-1)
     ap.add_argument("--K", type=int, default=0, help="override the config's K (e.g. 100 for SIFT1M)")
     ap.add_argument("--target-recall", type=float, default=0.95)
     ap.add_argument("--queue-len", type=int, default=0, help="skip the sweep")
@@ -196,6 +199,8 @@ def profiled_traffic(config_key: str):
 
 # ------------------------------------------------------------------ workload
 GRAPH_BUILDERS = ("auto", "batched", "exact")
+# song_build_graph_batched parameters of the bench's graph (override: --build-*)
+BUILD = {"prefix": 1 << 16, "queue_len": 64, "batch_shift": 1}
 
 
 def default_graph(cfg):
@@ -214,8 +219,8 @@ def build_graph_for(x, cfg, graph="auto"):
         graph = default_graph(cfg)
     if graph == "exact":
         return song.build_graph(x, cfg.degree, cfg.metric)
-    return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=1 << 16, queue_len=64,
-                                    batch_shift=1)
+    return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=BUILD["prefix"],
+                                    queue_len=BUILD["queue_len"], batch_shift=BUILD["batch_shift"])
 
 
 def build_workload(cfg, device, rank, log, cache="", graph="auto"):
@@ -544,6 +549,12 @@ def run_reference(args, ws, rank, local, log):
 
 def main():
     args = parse()
+    if args.build_prefix:
+        BUILD["prefix"] = args.build_prefix
+    if args.build_queue_len:
+        BUILD["queue_len"] = args.build_queue_len
+    if args.build_shift >= 0:
+        BUILD["batch_shift"] = args.build_shift
     if args.impl == "reference":
         # this tier's reference arm is the CPU oracle: rank 0 alone runs it
         ws = int(os.environ.get("WORLD_SIZE", "1"))

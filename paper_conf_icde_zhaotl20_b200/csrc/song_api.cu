@@ -135,6 +135,7 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_gtab);
   cudaFree(ix->d_R);
   cudaFree(ix->d_centroid);
+  cudaFreeHost(ix->h_status);
   cudaFree(ix->d_bins);
   cudaFree(ix->d_order);
   cudaFree(ix->d_qbin);
@@ -789,18 +790,22 @@ int song_search_codes_ex(song_index* ix, const song_search_params* p, const uint
                         counters_out, (cudaStream_t)stream);
 }
 
-int song_index_last_status(song_index* ix) {
-  if (!ix) return fail(SONG_EINVAL, "NULL index");
-  CUDA_TRY(cudaStreamSynchronize(ix->last_stream));
-  int st = 0;
-  CUDA_TRY(cudaMemcpy(&st, ix->d_status, sizeof st, cudaMemcpyDeviceToHost));
-  CUDA_TRY(cudaMemset(ix->d_status, 0, sizeof st));
+static int status_code(int st) {
   if (st & song::STATUS_BAD_INPUT) return fail(SONG_EINVAL, "a query had a non-finite value");
   if (st & song::STATUS_ITER_CAP) return fail(SONG_EITERCAP, "a query reached max_iters");
   if (st & song::STATUS_TABLE_FULL)
     return fail(SONG_EUNSUPPORTED, "a query filled half of its global visited table; raise "
                                    "table_log2");
   return SONG_OK;
+}
+
+int song_index_last_status(song_index* ix) {
+  if (!ix) return fail(SONG_EINVAL, "NULL index");
+  CUDA_TRY(cudaStreamSynchronize(ix->last_stream));
+  int st = 0;
+  CUDA_TRY(cudaMemcpy(&st, ix->d_status, sizeof st, cudaMemcpyDeviceToHost));
+  CUDA_TRY(cudaMemset(ix->d_status, 0, sizeof st));
+  return status_code(st);
 }
 
 int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int32_t queue_len,
@@ -845,7 +850,12 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
   if (rc) return rc;
   CUDA_TRY(cudaMemcpyAsync(ids_out, ix->d_ids, obytes, cudaMemcpyDeviceToHost, st));
   CUDA_TRY(cudaMemcpyAsync(dists_out, ix->d_dists, obytes, cudaMemcpyDeviceToHost, st));
-  return song_index_last_status(ix);
+  // the status word rides the same stream (one synchronisation per call)
+  if (!ix->h_status) CUDA_TRY(cudaMallocHost(&ix->h_status, sizeof(int)));
+  CUDA_TRY(cudaMemcpyAsync(ix->h_status, ix->d_status, sizeof(int), cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaMemsetAsync(ix->d_status, 0, sizeof(int), st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  return status_code(*ix->h_status);
 }
 
 int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,

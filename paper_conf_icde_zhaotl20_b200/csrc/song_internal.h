@@ -42,6 +42,7 @@ struct song_index {
   int32_t* d_order = nullptr;          // [nq] ticket -> query
   uint16_t* d_qbin = nullptr;          // [nq] bin of each query
   size_t cap_order = 0;
+  int* h_status = nullptr;             // pinned: song_search's status read-back
 };
 
 namespace song {

@@ -34,7 +34,13 @@ def main():
     res = {"config": cfg.name, "search_metric": cfg.metric}
     for gm in a.metrics.split(","):
         t = time.time()
-        if gm.endswith("-noheur"):  # torch tooling, plain NSW lists (no heuristic)
+        if gm.startswith("xbox"):  # MIPS -> L2 reduction: [x, sqrt(M^2 - |x|^2)], L2 graph
+            nrm2 = (x * x).sum(1)
+            xa = torch.cat([x, (nrm2.max() - nrm2).clamp_min(0).sqrt()[:, None]], 1).contiguous()
+            adj = (song.build_graph_batched(xa, cfg.degree, "l2", prefix=1 << 16, queue_len=64)
+                   if gm == "xbox-batched" else song.build_graph(xa, cfg.degree, "l2"))
+            del xa
+        elif gm.endswith("-noheur"):  # torch tooling, plain NSW lists (no heuristic)
             from workloads.graph import build_graph as tool_build
             adj = tool_build(x, cfg.degree, gm[:-len("-noheur")], heuristic=False)
         else:
