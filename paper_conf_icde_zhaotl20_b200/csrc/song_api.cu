@@ -221,7 +221,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   // Hamming codes: NCH = 16 B chunks per code (4 words), no row stage
   s.nch = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
-  const int rows = s.nch >= 8 ? 4 : std::min(32 / s.nch, SONG_STAGE_ROWS);  // StageRows<NCH>::R
+  const int rows = s.nch >= 2 ? 4 : SONG_STAGE_ROWS;  // StageRows<NCH>::R
   s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
