@@ -338,6 +338,21 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.steps = p->steps > 1 ? p->steps : 1;
   int warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
   while (warps > 1 && (size_t)sh.warp_bytes * warps > 200 * 1024) warps >>= 1;
+  if (p->warps_per_block <= 0 && sh.warp_bytes > 16 * 1024) {
+    // shared-memory-bound queue lengths: the CTA size that keeps the most warps
+    // resident (227 KB per SM; e.g. 73 KB per warp at L = 1536: 1-warp CTAs
+    // hold 3 warps per SM where 2-warp CTAs hold 2)
+    const size_t sm = 227 * 1024;
+    int best = 0;
+    for (int w = 4; w >= 1; w >>= 1) {
+      const size_t cta = (size_t)sh.warp_bytes * w + 1024;  // + the per-CTA reservation
+      const int res = cta <= sm ? (int)(sm / cta) * w : 0;
+      if (res > best) {
+        best = res;
+        warps = w;
+      }
+    }
+  }
   if ((size_t)sh.warp_bytes * warps > 227 * 1024)
     return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
                 p->queue_len, sh.warp_bytes);
