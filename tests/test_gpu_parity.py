@@ -402,6 +402,28 @@ def test_sift1m_full_size_sampled_parity():
     assert all(len(set(r)) == cfg.K for r in ii)
 
 
+@pytest.mark.parametrize("visited,steps,L", [("bloom", 1, 48), ("cuckoo", 1, 48),
+                                             ("hashtable-sel", 1, 48), ("hash", 2, 48),
+                                             ("hash", 1, 600)])
+def test_schedule_other_paths(sift100k, visited, steps, L):
+    """Outlier-first order on the other kernel variants (Bloom / Cuckoo / global
+    hash, multi-step probing, shared-memory queues): identical to batch order."""
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    qq = q.repeat(8, 1).contiguous()  # 4000 queries > 148 x 24 resident warps
+    res = []
+    for sched in ("batch", "outlier_first"):
+        ids, d, c = idx.search(qq, params=s.Params(K=cfg.K, queue_len=L, visited=visited,
+                                                   steps=steps, schedule=sched), counters=True)
+        torch.cuda.synchronize()
+        idx.last_status()
+        res.append((ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy()))
+    for a, b in zip(*res):
+        np.testing.assert_array_equal(a, b)
+    idx.close()
+
+
 @pytest.mark.parametrize("name,L", [("sift1m", 48), ("glove200", 64), ("nytimes256", 64)])
 def test_schedule_never_changes_results(name, L):
     """The outlier-first ticket order (song_search_params.schedule) only moves
