@@ -460,3 +460,31 @@ def test_schedule_never_changes_results(name, L):
                                 None, None)
     assert rc == -1 and b"schedule" in s.lib().song_last_error()
     idx.close()
+
+
+@pytest.mark.parametrize("dim", [1020, 1024])  # SONG_MAX_DIM: 8 chunks per lane, ragged last one
+def test_max_dim_exact(dim):
+    x, adj, q = small_random(n=2000, dim=dim)
+    s = song()
+    idx = s.SongIndex(x, adj)
+    for visited in ("hash", "bloom"):
+        g = gpu_search(idx, q, 10, 40, visited)
+        o = oracle.search(x, adj, q, 10, 40, **oracle_kw(visited, 40))
+        assert_exact(g, o)
+    idx.close()
+
+
+def test_single_vertex_and_isolated_entry():
+    """n = 1 (the entry is the only vertex), and an entry whose row is all
+    padding: one distance, one expansion, the rest of the output padded."""
+    s = song()
+    x = np.array([[3.0, 4.0]], np.float32)
+    idx = s.SongIndex(x, np.full((1, 4), -1, np.int32))
+    g = gpu_search(idx, np.zeros((2, 2), np.float32), 3, 4)
+    o = oracle.search(x, np.full((1, 4), -1, np.int32), np.zeros((2, 2), np.float32), 3, 4,
+                      **oracle_kw("hash", 4))
+    assert_exact(g, o)
+    assert (g[0][:, 0] == 0).all() and (g[0][:, 1:] == -1).all()
+    assert (g[1][:, 0] == 25.0).all() and np.isinf(g[1][:, 1:]).all()
+    assert (g[2] == [[1, 1]]).all()
+    idx.close()
