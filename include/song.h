@@ -292,6 +292,16 @@ int song_build_graph_batched(const float* vectors, int64_t n, int32_t dim, song_
                              int32_t degree, int32_t prefix, int32_t queue_len,
                              int32_t batch_shift, int32_t* adjacency_out, void* stream);
 
+/* R15 steps 2-4 (backward lists, candidates, HNSW heuristic with refill) on
+ * caller-given forward lists: fwd_ids / fwd_dists DEVICE [n][degree] (each row
+ * ascending by (dist, id), -1 past its entries, distances in the search's
+ * definition), e.g. kNN lists from another builder or a refinement search.
+ * Same arguments, scratch and errors as song_build_graph (+ SONG_EINVAL for
+ * NULL lists). */
+int song_build_graph_from_forward(const float* vectors, int64_t n, int32_t dim,
+                                  song_metric metric, int32_t degree, const int32_t* fwd_ids,
+                                  const float* fwd_dists, int32_t* adjacency_out, void* stream);
+
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);
 

@@ -315,3 +315,29 @@ extern "C" int song_build_graph_batched(const float* vectors, int64_t n, int32_t
   G_TRY(cudaStreamSynchronize(st));
   return SONG_OK;
 }
+
+extern "C" int song_build_graph_from_forward(const float* vectors, int64_t n, int32_t dim,
+                                             song_metric metric, int32_t degree,
+                                             const int32_t* fwd_ids, const float* fwd_dists,
+                                             int32_t* adjacency_out, void* stream) {
+  int rc = check_build_args(vectors, n, dim, metric, degree, adjacency_out);
+  if (rc) return rc;
+  if (!fwd_ids || !fwd_dists) return fail(SONG_EINVAL, "NULL forward lists");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int D = degree;
+  const int met = metric == SONG_L2 ? 0 : metric == SONG_IP ? 1 : 2;
+  Scratch s;
+  float* norms = nullptr;
+  const float* x = nullptr;
+  uint64_t* fkeys = nullptr;
+  if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
+  G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
+  const int kb = (int)std::min<int64_t>((n * D + 255) / 256, 148 * 32);
+  keys_from_results_kernel<<<kb, 256, 0, st>>>(fwd_ids, fwd_dists, n * D, fkeys);
+  G_TRY(cudaGetLastError());
+  Finish f;
+  G_TRY(f.alloc(s, n, D, st));
+  if ((rc = finish_graph(x, n, dim, met, D, norms, fkeys, f, adjacency_out, st))) return rc;
+  G_TRY(cudaStreamSynchronize(st));
+  return SONG_OK;
+}

@@ -33,7 +33,7 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
-            "song_search_codes_ex", "song_build_graph", "song_build_graph_batched"]
+            "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward"]
 
 
 class SongError(RuntimeError):
@@ -92,6 +92,7 @@ def lib():
         L.song_search_codes_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
         L.song_build_graph.argtypes = [P, i64, i32, i32, i32, P, P]
         L.song_build_graph_batched.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, P, P]
+        L.song_build_graph_from_forward.argtypes = [P, i64, i32, i32, i32, P, P, P, P]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -100,7 +101,8 @@ def lib():
                      "song_index_get_info", "song_search", "song_search_ex",
                      "song_index_last_status", "song_merge_topk", "song_rp_encode",
                      "song_index_create_codes", "song_index_create_rp",
-                     "song_search_codes_ex", "song_build_graph", "song_build_graph_batched"):
+                     "song_search_codes_ex", "song_build_graph", "song_build_graph_batched",
+                     "song_build_graph_from_forward"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -356,6 +358,22 @@ def build_graph_batched(vectors, degree: int = 32, metric: str = "l2", prefix: i
             ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1], METRICS[metric], degree,
             int(prefix), int(queue_len), int(batch_shift), ctypes.c_void_p(adj.data_ptr()),
             _stream_ptr(v.device)))
+    return adj
+
+
+def build_graph_from_forward(vectors, fwd_ids, fwd_dists, metric: str = "l2"):
+    """song_build_graph_from_forward: R15 steps 2-4 on given forward lists
+    (CUDA tensors [n, degree], rows ascending by (dist, id), -1 padded)."""
+    torch = _torch()
+    v = vectors.contiguous().float()
+    fi = fwd_ids.to(torch.int32).contiguous()
+    fd = fwd_dists.to(torch.float32).contiguous()
+    adj = torch.empty(fi.shape, dtype=torch.int32, device=v.device)
+    with torch.cuda.device(v.device):
+        _check(lib().song_build_graph_from_forward(
+            ctypes.c_void_p(v.data_ptr()), v.shape[0], v.shape[1], METRICS[metric], fi.shape[1],
+            ctypes.c_void_p(fi.data_ptr()), ctypes.c_void_p(fd.data_ptr()),
+            ctypes.c_void_p(adj.data_ptr()), _stream_ptr(v.device)))
     return adj
 
 

@@ -160,3 +160,21 @@ def test_batched_errors():
     for kw in (dict(prefix=0), dict(queue_len=4), dict(batch_shift=17)):
         with pytest.raises(s.SongError):
             s.build_graph_batched(x, 8, **kw)
+
+
+def test_from_forward_bit_exact():
+    """song_build_graph_from_forward (R15 steps 2-4 on given lists) against the
+    oracle's, on the oracle's own exact forward lists and on lists with gaps."""
+    x = og._int_data(2500, 24, 21)
+    fi, fd = oracle.forward_lists(x, 16, nthreads=8)
+    fi[::7, 5:] = -1  # shorter lists on some rows
+    fd[::7, 5:] = np.inf
+    want = oracle.build_graph_from_forward(x, fi, fd, nthreads=8)
+    s = song()
+    got = s.build_graph_from_forward(torch.as_tensor(x, device="cuda"),
+                                     torch.as_tensor(fi, device="cuda"),
+                                     torch.as_tensor(fd, device="cuda"))
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(got.cpu().numpy(), want)
+    np.testing.assert_array_equal(oracle.build_graph_from_forward(x, *oracle.forward_lists(x, 16)),
+                                  oracle.build_graph(x, 16))
