@@ -417,7 +417,12 @@ def run_song(args, ws, rank, local, log):
         "e2e": {"value": round(e2e_value, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(qh.numel() * 4),
                 "d2h_bytes_per_step": int(ih.numel() * 4 + dh.numel() * 4),
-                "host_results_match_device": host_ok},
+                "host_results_match_device": host_ok,
+                # wall-clock per call (value above = steps / their sum): host
+                # jitter on the box shows up as max >> median
+                "ms_per_step": {"min": round(min(e2e_s) * 1e3, 4),
+                                "median": round(sorted(e2e_s)[len(e2e_s) // 2] * 1e3, 4),
+                                "max": round(max(e2e_s) * 1e3, 4)}},
         "clocks": clk.summary(),
         # per step: the search kernel, plus the two outlier-first scheduling
         # kernels (order keys + scatter) when the batch outnumbers the resident
