@@ -27,8 +27,16 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-GRID = [10, 12, 16, 20, 24, 32, 40, 48, 64, 80, 96, 128, 160, 192, 256, 384, 512, 768,
-        1024, 1536, 2048]
+GRID = [10, 12, 16, 20, 24, 28, 32, 36, 40, 44, 48, 56, 64, 72, 80, 96, 112, 128, 144, 160,
+        192, 224, 256, 320, 384, 448, 512, 640, 768, 896, 1024, 1280, 1536, 2048]
+
+
+def grid_for(K):
+    """queue_len candidates of the operating-point sweep: K itself, then the
+    grid above it (the smallest with recall >= target is the operating point)."""
+    return sorted({K, *(g for g in GRID if g >= K)})
+
+
 METRIC = "queries/sec at recall@10=0.95 (SIFT1M-shaped), 1/2/4/8 B200; % HBM roofline"
 
 
@@ -185,6 +193,27 @@ def measured_peak_hbm():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def gpu_local_cpus(dev: int) -> set:
+    """Host cores on the GPU's NUMA node (sysfs local_cpulist of its PCI
+    function), or an empty set when unknown."""
+    import torch
+    try:
+        p = torch.cuda.get_device_properties(dev)
+        bus = f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+        with open(f"/sys/bus/pci/devices/{bus}/local_cpulist") as f:
+            text = f.read().strip()
+    except (OSError, AttributeError, RuntimeError, ValueError):
+        return set()
+    cpus = set()
+    for part in text.split(","):
+        if "-" in part:
+            a, b = part.split("-")
+            cpus.update(range(int(a), int(b) + 1))
+        elif part:
+            cpus.add(int(part))
+    return cpus
+
+
 def profiled_traffic(config_key: str):
     """dram bytes per launch from a committed `ncu --set full` capture."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
@@ -304,9 +333,8 @@ def run_song(args, ws, rank, local, log):
     sweep = []
     L_op = args.queue_len
     if not L_op:
-        for L in GRID:
-            if L < cfg.K:
-                continue
+        # queue_len = K itself first (K = 100 is not on the grid)
+        for L in grid_for(cfg.K):
             ids, _ = idx.search(q0, params=params(L))
             r = recall_t(ids, truth0)
             sweep.append((L, round(r, 4)))
@@ -371,10 +399,16 @@ def run_song(args, ws, rank, local, log):
     if args.profile:
         log(f"profile run: {step_ms}")
         return None
-    # ---- end to end through the C ABI's host-buffer entry point
-    qh = q.cpu().pin_memory()
-    ih = torch.empty((nq, K), dtype=torch.int32).pin_memory()
-    dh = torch.empty((nq, K), dtype=torch.float32).pin_memory()
+    # ---- end to end through the C ABI's host-buffer entry point, from the
+    # host cores (and pinned memory) on the GPU's own NUMA node
+    all_cpus = os.sched_getaffinity(0)
+    near = gpu_local_cpus(torch.cuda.current_device()) & all_cpus
+    if near:
+        os.sched_setaffinity(0, near)
+    qh = torch.empty(q.shape, dtype=torch.float32, pin_memory=True)
+    qh.copy_(q.cpu())
+    ih = torch.empty((nq, K), dtype=torch.int32, pin_memory=True)
+    dh = torch.empty((nq, K), dtype=torch.float32, pin_memory=True)
     for _ in range(max(1, args.warmup)):
         idx.search_host_into(qh, K, L_op, ih, dh)
     e2e_s = []
@@ -388,6 +422,7 @@ def run_song(args, ws, rank, local, log):
     e2e_total = allreduce_max(sum(e2e_s), ws)
     e2e_value = ws * nq * args.steps / e2e_total
     host_ok = bool((ih.numpy() == out[0].cpu().numpy()).all())
+    os.sched_setaffinity(0, all_cpus)  # the CPU baseline uses every core
 
     result = {
         "metric": metric_name(cfg, args.target_recall), "value": round(value, 1), "unit": "queries/s", "n_gpus": ws,
@@ -418,6 +453,8 @@ def run_song(args, ws, rank, local, log):
                 "h2d_bytes_per_step": int(qh.numel() * 4),
                 "d2h_bytes_per_step": int(ih.numel() * 4 + dh.numel() * 4),
                 "host_results_match_device": host_ok,
+                "host_cpus": f"{len(near)} GPU-local cores (NUMA node of the GPU)" if near
+                             else f"{len(all_cpus)} cores (GPU locality unknown)",
                 # wall-clock per call (value above = steps / their sum): host
                 # jitter on the box shows up as max >> median
                 "ms_per_step": {"min": round(min(e2e_s) * 1e3, 4),
@@ -509,9 +546,7 @@ def run_reference(args, ws, rank, local, log):
     L_op = args.queue_len
     sweep = []
     if not L_op:  # same operating-point rule as the song arm, on the same full batch
-        for L in GRID:
-            if L < cfg.K:
-                continue
+        for L in grid_for(cfg.K):
             ids, _, _, _ = oracle.search(xn, an, qn, cfg.K, L, metric=m, nthreads=cores,
                                          **oracle_mode(L))
             r = oracle.recall(ids, truth)
