@@ -5,6 +5,7 @@ copy of the query batch alone, the DtoH of the results alone, the device step
 
     python tools/e2e_probe.py
 """
+import json
 import os
 import sys
 import time
@@ -51,7 +52,48 @@ def main():
     p = song.Params(K=10, queue_len=L)
     res["device_step_wall_ms"] = wall(lambda: idx.search(q, params=p, out=out))
     res["song_search_ms"] = wall(lambda: idx.search_host_into(qh, 10, L, ih, dh))
-    print(res)
+    # as bench.py's e2e loop: a 512 MiB L2 flush + synchronize before each call
+    flush = torch.empty(128 << 20, dtype=torch.float32, device=dev)
+
+    def flushed(fn, n=20):
+        ts = []
+        for i in range(n + 3):
+            flush.zero_()
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            fn()
+            torch.cuda.synchronize()
+            if i >= 3:
+                ts.append(time.perf_counter() - t)
+        return [round(float(np.percentile(ts, k)) * 1e3, 4) for k in (0, 50, 100)]
+
+    res["device_step_wall_flushed_ms_min_med_max"] = flushed(
+        lambda: idx.search(q, params=p, out=out))
+    res["song_search_flushed_ms_min_med_max"] = flushed(
+        lambda: idx.search_host_into(qh, 10, L, ih, dh))
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+
+    def dev_timed_call():
+        ev[0].record()
+        idx.search_host_into(qh, 10, L, ih, dh)
+        ev[1].record()
+
+    # the call on the device clock (events on torch's stream bracket the
+    # library's stream work because song_search synchronizes before returning)
+    ts = []
+    for i in range(23):
+        flush.zero_()
+        torch.cuda.synchronize()
+        dev_timed_call()
+        torch.cuda.synchronize()
+        if i >= 3:
+            ts.append(ev[0].elapsed_time(ev[1]))
+    res["song_search_flushed_event_ms_min_med_max"] = [round(float(np.percentile(ts, k)), 4)
+                                                       for k in (0, 50, 100)]
+    print(json.dumps(res))
+    if len(sys.argv) > 1:
+        with open(sys.argv[1], "w") as f:
+            json.dump(res, f, indent=1)
 
 
 if __name__ == "__main__":
