@@ -1,0 +1,30 @@
+"""Host logic of bench.py that decides what is measured (no GPU): the
+operating-point grid and the GPU-local host-core parsing."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import bench  # noqa: E402
+
+
+def test_grid_starts_at_K_and_is_ascending():
+    for K in (1, 10, 100, 127, 1000):
+        g = bench.grid_for(K)
+        assert g[0] == K
+        assert g == sorted(set(g))
+        assert all(L >= K for L in g)
+        # every grid point at or above K is offered
+        assert set(L for L in bench.GRID if L >= K) <= set(g)
+
+
+def test_grid_for_K10_is_the_plain_grid():
+    assert bench.grid_for(10) == bench.GRID
+
+
+def test_gpu_local_cpus_without_gpu_is_empty():
+    import torch
+    if torch.cuda.is_available():
+        return
+    assert bench.gpu_local_cpus(0) == set()
