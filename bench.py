@@ -230,14 +230,26 @@ def profiled_traffic(config_key: str):
 GRAPH_BUILDERS = ("auto", "batched", "exact")
 # song_build_graph_batched parameters of the bench's graph (override: --build-*)
 BUILD = {"prefix": 1 << 16, "queue_len": 64, "batch_shift": 1}
+# per-config builder parameters (measured, profiles/r01t_build_sweep_nyt.txt:
+# NYTimes L 160 -> 144 at recall 0.95); CLI --build-* still win
+BUILD_FOR = {"nytimes256": {"queue_len": 128, "batch_shift": 2}}
+_BUILD_CLI = set()
+
+
+def build_params(cfg):
+    p = dict(BUILD)
+    p.update({k: v for k, v in BUILD_FOR.get(cfg.name, {}).items() if k not in _BUILD_CLI})
+    return p
 
 
 def default_graph(cfg):
-    """Measured per metric: batched insertion (R16) gives the
-    L2 / cosine workloads better graphs than exact insertion (SIFT1M L 48 -> 32,
-    NYTimes 768 -> 160 at recall 0.95); on the IP workload its search-built
-    forward lists cap recall near 0.90, so IP keeps exact insertion (R15)."""
-    return "exact" if cfg.metric == "ip" else "batched"
+    """Measured per workload: batched insertion (R16) gives the
+    SIFT / cosine workloads better graphs than exact insertion (SIFT1M L 48 -> 32,
+    NYTimes 768 -> 144 at recall 0.95); on the IP workload its search-built
+    forward lists cap recall near 0.90, and on the 960-d GIST workload exact
+    insertion needs L 28 where R16 needs 40 (profiles/r01t_bench_gist1m_exact.log),
+    so those keep exact insertion (R15)."""
+    return "exact" if cfg.metric == "ip" or cfg.dim >= 512 else "batched"
 
 
 def build_graph_for(x, cfg, graph="auto"):
@@ -248,8 +260,9 @@ def build_graph_for(x, cfg, graph="auto"):
         graph = default_graph(cfg)
     if graph == "exact":
         return song.build_graph(x, cfg.degree, cfg.metric)
-    return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=BUILD["prefix"],
-                                    queue_len=BUILD["queue_len"], batch_shift=BUILD["batch_shift"])
+    b = build_params(cfg)
+    return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=b["prefix"],
+                                    queue_len=b["queue_len"], batch_shift=b["batch_shift"])
 
 
 def build_workload(cfg, device, rank, log, cache="", graph="auto"):
@@ -605,10 +618,13 @@ def main():
     args = parse()
     if args.build_prefix:
         BUILD["prefix"] = args.build_prefix
+        _BUILD_CLI.add("prefix")
     if args.build_queue_len:
         BUILD["queue_len"] = args.build_queue_len
+        _BUILD_CLI.add("queue_len")
     if args.build_shift >= 0:
         BUILD["batch_shift"] = args.build_shift
+        _BUILD_CLI.add("batch_shift")
     if args.impl == "reference":
         # this tier's reference arm is the CPU oracle: rank 0 alone runs it
         ws = int(os.environ.get("WORLD_SIZE", "1"))

@@ -28,3 +28,14 @@ def test_gpu_local_cpus_without_gpu_is_empty():
     if torch.cuda.is_available():
         return
     assert bench.gpu_local_cpus(0) == set()
+
+
+def test_graph_choice_and_builder_params_per_config():
+    from workloads.synth import CONFIGS
+    assert bench.default_graph(CONFIGS["sift1m"]) == "batched"
+    assert bench.default_graph(CONFIGS["nytimes256"]) == "batched"
+    assert bench.default_graph(CONFIGS["gist1m"]) == "exact"
+    assert bench.default_graph(CONFIGS["glove200"]) == "exact"
+    assert bench.build_params(CONFIGS["sift1m"]) == bench.BUILD
+    nyt = bench.build_params(CONFIGS["nytimes256"])
+    assert nyt["queue_len"] == 128 and nyt["batch_shift"] == 2
