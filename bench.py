@@ -229,10 +229,12 @@ def profiled_traffic(config_key: str):
 # ------------------------------------------------------------------ workload
 GRAPH_BUILDERS = ("auto", "batched", "exact")
 # song_build_graph_batched parameters of the bench's graph (override: --build-*)
-BUILD = {"prefix": 1 << 16, "queue_len": 64, "batch_shift": 1}
-# per-config builder parameters (measured, profiles/r01t_build_sweep_nyt.txt:
-# NYTimes L 160 -> 144 at recall 0.95); CLI --build-* still win
-BUILD_FOR = {"nytimes256": {"queue_len": 128, "batch_shift": 2}}
+# (measured: profiles/r01u_build_sweep_sift.txt, r01t_build_sweep_nyt.txt —
+# build queue_len 128 with batches of m/4 gives SIFT1M L 32 -> 28 and NYTimes
+# L 160 -> 144 at recall 0.95 against queue_len 64, batches of m/2)
+BUILD = {"prefix": 1 << 16, "queue_len": 128, "batch_shift": 2}
+# per-config overrides of BUILD (none today); CLI --build-* still win
+BUILD_FOR = {}
 _BUILD_CLI = set()
 
 
@@ -254,7 +256,7 @@ def default_graph(cfg):
 
 def build_graph_for(x, cfg, graph="auto"):
     """The bench's graph: song_build_graph_batched (reading R16; prefix 2^16
-    rows exact, batches of m/2 searched at L = 64) or song_build_graph (R15)."""
+    rows exact, batches of m/4 searched at L = 128) or song_build_graph (R15)."""
     from paper_conf_icde_zhaotl20_b200 import song
     if graph == "auto":
         graph = default_graph(cfg)

@@ -36,6 +36,7 @@ def test_graph_choice_and_builder_params_per_config():
     assert bench.default_graph(CONFIGS["nytimes256"]) == "batched"
     assert bench.default_graph(CONFIGS["gist1m"]) == "exact"
     assert bench.default_graph(CONFIGS["glove200"]) == "exact"
-    assert bench.build_params(CONFIGS["sift1m"]) == bench.BUILD
-    nyt = bench.build_params(CONFIGS["nytimes256"])
-    assert nyt["queue_len"] == 128 and nyt["batch_shift"] == 2
+    for name in ("sift1m", "nytimes256"):
+        b = bench.build_params(CONFIGS[name])
+        assert b == bench.BUILD
+        assert b["queue_len"] == 128 and b["batch_shift"] == 2 and b["prefix"] == 1 << 16
