@@ -101,8 +101,8 @@ def main():
     ap.add_argument("--n", type=int, default=100_000_000)
     ap.add_argument("--nq", type=int, default=10_000)
     ap.add_argument("--prefix", type=int, default=1 << 16)
-    ap.add_argument("--build-queue-len", type=int, default=64)
-    ap.add_argument("--batch-shift", type=int, default=1)
+    ap.add_argument("--build-queue-len", type=int, default=128)
+    ap.add_argument("--batch-shift", type=int, default=2)
     ap.add_argument("--compare-exact", action="store_true")
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--parity-sample", type=int, default=0,
