@@ -153,6 +153,35 @@ typedef struct song_index_info {
 /* Fill p with the library defaults for (K, queue_len). Never fails. */
 void song_default_params(song_search_params* p, int32_t K, int32_t queue_len);
 
+/* What song_search_ex would run for `params` on an index of `dim` dimensions
+ * and `metric` (SONG_HAMMING: dim = code words, bits / 32) — the resolved
+ * data-structure sizes and launch shape.  Pure host computation: it never
+ * touches a device, so it is callable without a GPU.  This is the single
+ * source of the library's defaults (tests, bench and tools read the lazy
+ * deletion capacity and the visited-table size from here rather than
+ * re-deriving them). */
+typedef struct song_search_plan {
+  int32_t visited_log2;    /* SONG_VISITED_HASH, _HASH_GLOBAL(_SEL): log2 table slots;
+                              BLOOM: log2 bits m (reading A11); CUCKOO: log2 buckets of
+                              4 fingerprints (reading R10) */
+  int32_t visited_cap;     /* SONG_VISITED_HASH: the capacity C of lazy deletion in effect
+                              (reading R14; the oracle's lazy_cap), or -1 for eager
+                              deletion (visited_cap = -1 or steps > 1); 0 for the other
+                              kinds */
+  int32_t queue_regs;      /* q and topk held in registers, queue_regs u64 per lane
+                              (queue_len <= 32 * queue_regs); 0 = shared-memory queues */
+  int32_t row_chunks;      /* 16 B chunks per lane of a staged row (NCH) */
+  int32_t smem_per_warp;   /* shared-memory bytes per warp */
+  int32_t warps_per_block; /* CTA size of the persistent grid (1 warp = 1 query) */
+  int32_t reserved[2];     /* 0 */
+} song_search_plan;
+
+/* Errors: SONG_EINVAL (NULL, bad params as song_search_ex would report them,
+ * except the entry range, which needs the index), SONG_EUNSUPPORTED (the
+ * sizes above the compiled maxima, shared-memory budget exceeded). */
+int song_search_plan_get(const song_search_params* params, int32_t dim, int32_t metric,
+                         song_search_plan* out);
+
 /* Create an index on the current CUDA device from HOST arrays (§IV-A, P:267,
  * graph and data are persisted in global memory before any query).
  *   vectors   [n][dim] fp32, host; copied (rows padded to 16 B; for
@@ -194,6 +223,11 @@ int song_search(song_index* idx, const float* queries, int64_t nq, int32_t K,
  * defines the roofline bytes.  A query with a non-finite value gets ids -1;
  * one that reaches max_iters returns its partial topk; both are reported by
  * song_index_last_status().
+ * Concurrency: the searches of one index share its work counter and status
+ * word, so the library orders them: a search enqueued on a stream other than
+ * the previous search's waits (cudaStreamWaitEvent) for that search to finish
+ * on the device.  Searches of distinct indexes run concurrently.  Host calls
+ * on one index must not race (one host thread at a time per index).
  * Errors detectable before launch: SONG_EINVAL, SONG_EUNSUPPORTED, SONG_ECUDA. */
 int song_search_ex(song_index* idx, const song_search_params* params,
                    const float* queries, int64_t nq, int32_t* ids_out, float* dists_out,
@@ -260,6 +294,11 @@ int song_search_codes_ex(song_index* idx, const song_search_params* params,
                          float* dists_out, int32_t* counters_out, void* stream);
 
 /* ---- graph construction (reading R15) ----
+ * All three builders first scan the rows on the device: a non-finite value is
+ * SONG_EINVAL.  Step 1's distance tiles run on the tensor cores (tcgen05
+ * kind::tf32) only when that is exact — every value an integer, dim *
+ * max|x|^2 < 2^24, rows 16 B aligned — and on fp32 FFMA tiles otherwise.
+ *
  * SONG searches pre-built NSW graphs; this builds one on the
  * device: forward lists F(i) = the `degree` nearest earlier vertices (exact
  * insertion NSW), backward lists B(j) = the `degree` nearest i with j in F(i),
@@ -296,8 +335,11 @@ int song_build_graph_batched(const float* vectors, int64_t n, int32_t dim, song_
  * caller-given forward lists: fwd_ids / fwd_dists DEVICE [n][degree] (each row
  * ascending by (dist, id), -1 past its entries, distances in the search's
  * definition), e.g. kNN lists from another builder or a refinement search.
- * Same arguments, scratch and errors as song_build_graph (+ SONG_EINVAL for
- * NULL lists). */
+ * The lists need not be earlier-only: the candidates C(v) = F(v) u B(v) are
+ * taken as a set of vertices (v itself dropped, an id in both lists kept once
+ * at its smaller key).  Same arguments, scratch and errors as
+ * song_build_graph, + SONG_EINVAL for NULL lists or an id outside [-1, n)
+ * (checked on the device before any work). */
 int song_build_graph_from_forward(const float* vectors, int64_t n, int32_t dim,
                                   song_metric metric, int32_t degree, const int32_t* fwd_ids,
                                   const float* fwd_dists, int32_t* adjacency_out, void* stream);

@@ -57,7 +57,10 @@
 //      1. forward F(i) = the D smallest keys (d(i, j), j) over j < i
 //         (exact-insertion NSW: each vertex links to its D nearest earlier ones);
 //      2. backward B(j) = the D smallest keys (d(i, j), i) over {i : j in F(i)};
-//      3. C(v) = F(v) u B(v) (disjoint: ids < v and > v) ascending by key;
+//      3. C(v) = F(v) u B(v) ascending by key, as a set of vertices: v itself
+//         is dropped and an id in both lists is kept once at its smaller key
+//         (a no-op for 1.'s earlier-only lists, where F(v) < v < B(v); caller-
+//         given kNN lists, song_build_graph_from_forward, can overlap);
 //      4. HNSW heuristic: walk C(v) in order, keep c while fewer than D are kept
 //         and d(c, k) > d(c, v) for every kept k ("closer to the base than to
 //         every kept neighbour"); then refill with the skipped candidates in
@@ -589,9 +592,18 @@ static void build_from_forward(const float* data, int64_t n, int32_t dim, int32_
   });
   // 3. + 4. candidates and the heuristic
   parallel([&](int64_t v) {
-    std::vector<Key> C = F[v];
-    C.insert(C.end(), B[v].begin(), B[v].end());
-    std::sort(C.begin(), C.end());
+    std::vector<Key> all = F[v];
+    all.insert(all.end(), B[v].begin(), B[v].end());
+    std::sort(all.begin(), all.end());
+    // C(v) = F(v) ∪ B(v) as a set of vertices (R15): v itself is not its own
+    // neighbour, and an id in both lists is kept once, at its smaller key
+    std::vector<Key> C;
+    for (const Key& k : all) {
+      if (k.id == (int32_t)v) continue;
+      bool seen = false;
+      for (const Key& c : C) seen = seen || c.id == k.id;
+      if (!seen) C.push_back(k);
+    }
     std::vector<int32_t> kept;
     std::vector<char> taken(C.size(), 0);
     for (size_t t = 0; t < C.size() && (int)kept.size() < D; ++t) {

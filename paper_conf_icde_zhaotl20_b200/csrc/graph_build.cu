@@ -46,6 +46,46 @@ __global__ void count_u64_kernel(const uint64_t* __restrict__ fkeys, int64_t ned
   }
 }
 
+// one pass over the builder's input rows: non-finite values (rejected),
+// whether every value is an integer, and the largest |value| (bits of a
+// non-negative float compare like ints) — the tensor-core Gram is taken only
+// when it is provably exact (forward_exact)
+struct RowScan {
+  unsigned long long nonfinite;
+  int non_integer;
+  unsigned max_abs_bits;
+};
+
+__global__ void scan_rows_kernel(const float* __restrict__ x, int64_t m, RowScan* out) {
+  unsigned long long bad = 0;
+  int nonint = 0;
+  unsigned mx = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const float v = x[i];
+    if (!isfinite(v)) {
+      ++bad;
+      continue;
+    }
+    nonint |= rintf(v) != v;
+    mx = max(mx, __float_as_uint(fabsf(v)));
+  }
+  if (bad) atomicAdd(&out->nonfinite, bad);
+  if (__syncthreads_or(nonint) && threadIdx.x == 0) atomicOr(&out->non_integer, 1);
+  for (int o = 16; o >= 1; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(&out->max_abs_bits, mx);
+}
+
+// forward-list ids given by the caller: in [-1, n)
+__global__ void check_ids_kernel(const int32_t* __restrict__ ids, int64_t m, int64_t n,
+                                 unsigned long long* bad) {
+  unsigned long long b = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x)
+    b += (ids[i] < -1 || ids[i] >= n);
+  if (b) atomicAdd(bad, b);
+}
+
 __global__ void narrow_kernel(const unsigned long long* a, int* b, int64_t n) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -135,24 +175,21 @@ int finish_graph(const float* x, int64_t n, int dim, int met, int D, const float
   return SONG_OK;
 }
 
-// R15 step 1 on rows [0, n): tensor cores (tcgen05, tf32) when that is exact
-// for the data (every value tf32-representable, rows 16 B aligned), else FFMA
+// R15 step 1 on rows [0, n): tensor cores (tcgen05, tf32) only when that is
+// provably exact — every value an integer with dim * max|x|^2 < 2^24, so every
+// product and partial sum is an integer below 2^24 and any summation order
+// gives the same fp32 result as the FFMA tiles and the oracle — else FFMA
 int forward_exact(const float* x, int64_t n, int dim, int met, bool cosine, int D,
-                  const float* norms, uint64_t* fkeys, Scratch& s, cudaStream_t st) {
+                  const float* norms, const RowScan& scan, uint64_t* fkeys, Scratch& s,
+                  cudaStream_t st) {
   using namespace song::graph;
-  bool use_tc = dim % 4 == 0 && !cosine;
+  float mx;
+  std::memcpy(&mx, &scan.max_abs_bits, sizeof mx);
+  bool use_tc = dim % 4 == 0 && !cosine && (reinterpret_cast<uintptr_t>(x) & 15) == 0 &&
+                !scan.non_integer && (double)dim * mx * mx < 16777216.0;
   const char* force = std::getenv("SONG_GRAPH_PATH");  // "simt" / "tc" (tests, A/B)
-  if (use_tc && !(force && std::strcmp(force, "tc") == 0)) {
-    int* d_flag = nullptr;
-    G_TRY(s.get(&d_flag, sizeof(int)));
-    G_TRY(cudaMemsetAsync(d_flag, 0, sizeof(int), st));
-    song::graph::tc::tf32_exact_kernel<<<592, 256, 0, st>>>(x, n * (int64_t)dim, d_flag);
-    G_TRY(cudaGetLastError());
-    int not_exact = 0;
-    G_TRY(cudaMemcpyAsync(&not_exact, d_flag, sizeof(int), cudaMemcpyDeviceToHost, st));
-    G_TRY(cudaStreamSynchronize(st));
-    use_tc = !not_exact;
-  }
+  if (force && std::strcmp(force, "tc") == 0)
+    use_tc = dim % 4 == 0 && !cosine && (reinterpret_cast<uintptr_t>(x) & 15) == 0;
   if (force && std::strcmp(force, "simt") == 0) use_tc = false;
   if (use_tc) {
     namespace tc = song::graph::tc;
@@ -171,6 +208,21 @@ int forward_exact(const float* x, int64_t n, int dim, int met, bool cosine, int 
     knn_prefix_kernel<<<(unsigned)nb, THREADS, 0, st>>>(x, n, dim, norms, met, D, fkeys);
     G_TRY(cudaGetLastError());
   }
+  return SONG_OK;
+}
+
+// scan the input rows (rejecting non-finite values: song.h, SONG_EINVAL)
+int scan_rows(const float* vectors, int64_t n, int dim, Scratch& s, RowScan* out,
+              cudaStream_t st) {
+  RowScan* d = nullptr;
+  G_TRY(s.get(&d, sizeof(RowScan)));
+  G_TRY(cudaMemsetAsync(d, 0, sizeof(RowScan), st));
+  scan_rows_kernel<<<592, 256, 0, st>>>(vectors, n * (int64_t)dim, d);
+  G_TRY(cudaGetLastError());
+  G_TRY(cudaMemcpyAsync(out, d, sizeof(RowScan), cudaMemcpyDeviceToHost, st));
+  G_TRY(cudaStreamSynchronize(st));
+  if (out->nonfinite)
+    return fail(SONG_EINVAL, "%llu non-finite vector values", out->nonfinite);
   return SONG_OK;
 }
 
@@ -231,10 +283,13 @@ extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, so
   float* norms = nullptr;
   const float* x = nullptr;
   uint64_t* fkeys = nullptr;
+  RowScan scan;
+  if ((rc = scan_rows(vectors, n, dim, s, &scan, st))) return rc;
   if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
   G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
   // 1. forward lists
-  if ((rc = forward_exact(x, n, dim, met, metric == SONG_COSINE, D, norms, fkeys, s, st))) return rc;
+  if ((rc = forward_exact(x, n, dim, met, metric == SONG_COSINE, D, norms, scan, fkeys, s, st)))
+    return rc;
   // 2. - 4.
   Finish f;
   G_TRY(f.alloc(s, n, D, st));
@@ -260,11 +315,14 @@ extern "C" int song_build_graph_batched(const float* vectors, int64_t n, int32_t
   float* norms = nullptr;
   const float* x = nullptr;
   uint64_t* fkeys = nullptr;
+  RowScan scan;
+  if ((rc = scan_rows(vectors, n, dim, s, &scan, st))) return rc;
   if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
   G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
   // 1. exact forward lists of the prefix (R15 step 1)
   const int64_t m0 = std::min<int64_t>(n, prefix);
-  if ((rc = forward_exact(x, m0, dim, met, metric == SONG_COSINE, D, norms, fkeys, s, st))) return rc;
+  if ((rc = forward_exact(x, m0, dim, met, metric == SONG_COSINE, D, norms, scan, fkeys, s, st)))
+    return rc;
   Finish f;
   G_TRY(f.alloc(s, n, D, st));
   if (m0 < n) {
@@ -308,7 +366,7 @@ extern "C" int song_build_graph_batched(const float* vectors, int64_t n, int32_t
     if (rc == SONG_OK) rc = song::view_status(view, &status, st);
     song::free_search_view(view);
     if (rc) return rc;
-    if (status & song::STATUS_BAD_INPUT) return fail(SONG_EINVAL, "vectors hold non-finite values");
+    if (status) return fail(SONG_ECUDA, "batch search status %d", status);
   }
   // 3. the graph on all rows
   if ((rc = finish_graph(x, n, dim, met, D, norms, fkeys, f, adjacency_out, st))) return rc;
@@ -330,6 +388,19 @@ extern "C" int song_build_graph_from_forward(const float* vectors, int64_t n, in
   float* norms = nullptr;
   const float* x = nullptr;
   uint64_t* fkeys = nullptr;
+  RowScan scan;
+  if ((rc = scan_rows(vectors, n, dim, s, &scan, st))) return rc;
+  {
+    unsigned long long* d_bad = nullptr;
+    G_TRY(s.get(&d_bad, sizeof *d_bad));
+    G_TRY(cudaMemsetAsync(d_bad, 0, sizeof *d_bad, st));
+    check_ids_kernel<<<592, 256, 0, st>>>(fwd_ids, n * (int64_t)D, n, d_bad);
+    G_TRY(cudaGetLastError());
+    unsigned long long bad = 0;
+    G_TRY(cudaMemcpyAsync(&bad, d_bad, sizeof bad, cudaMemcpyDeviceToHost, st));
+    G_TRY(cudaStreamSynchronize(st));
+    if (bad) return fail(SONG_EINVAL, "%llu forward-list ids outside [-1, n)", bad);
+  }
   if ((rc = prepare_rows(vectors, n, dim, metric, s, &norms, &x, st))) return rc;
   G_TRY(s.get(&fkeys, n * (int64_t)D * sizeof(uint64_t)));
   const int kb = (int)std::min<int64_t>((n * D + 255) / 256, 148 * 32);

@@ -231,11 +231,41 @@ __global__ void __launch_bounds__(PT) prune_kernel(const float* __restrict__ x, 
         a0 = low ? umin64(a0, o0) : umax64(a0, o0);
         a1 = low ? umin64(a1, o1) : umax64(a1, o1);
       }
-      cand[lane] = a0;
-      cand[lane + 32] = a1;
-      const int c = __popc(__ballot_sync(FULL, a0 != KEY_MAX)) + __popc(__ballot_sync(FULL, a1 != KEY_MAX));
-      cid[lane] = a0 != KEY_MAX ? key_id(a0) : 0;
-      cid[lane + 32] = a1 != KEY_MAX ? key_id(a1) : 0;
+      // C(v) as a set of vertices: drop v itself and every repeat of an id
+      // after its first (smallest-key) occurrence — F(v) and B(v) overlap
+      // when the forward lists are not earlier-only (kNN lists given to
+      // song_build_graph_from_forward); a no-op for the builders' own lists
+      const int i0 = a0 != KEY_MAX ? key_id(a0) : -1, i1 = a1 != KEY_MAX ? key_id(a1) : -1;
+      cid[lane] = i0;
+      cid[lane + 32] = i1;
+      __syncwarp();
+      bool k0 = i0 >= 0 && i0 != (int)v, k1 = i1 >= 0 && i1 != (int)v;
+      for (int t = 0; t < PC; ++t) {
+        const int o = cid[t];
+        k0 = k0 && !(t < lane && o == i0);
+        k1 = k1 && !(t < lane + 32 && o == i1);
+      }
+      const unsigned m0 = __ballot_sync(FULL, k0), m1 = __ballot_sync(FULL, k1);
+      const unsigned lt = lanemask_lt();
+      __syncwarp();
+      if (k0) {
+        cand[__popc(m0 & lt)] = a0;
+        cid[__popc(m0 & lt)] = i0;
+      }
+      if (k1) {
+        cand[__popc(m0) + __popc(m1 & lt)] = a1;
+        cid[__popc(m0) + __popc(m1 & lt)] = i1;
+      }
+      const int c = __popc(m0) + __popc(m1);
+      __syncwarp();
+      if (lane >= c) {
+        cand[lane] = KEY_MAX;
+        cid[lane] = 0;
+      }
+      if (lane + 32 >= c) {
+        cand[lane + 32] = KEY_MAX;
+        cid[lane + 32] = 0;
+      }
       if (lane == 0) ncand = c;
     }
     __syncthreads();

@@ -256,15 +256,6 @@ __global__ void __launch_bounds__(THREADS, 1)
   }
 }
 
-// 1 if every value is exactly representable in tf32 (low 13 mantissa bits 0)
-__global__ void tf32_exact_kernel(const float* __restrict__ x, int64_t m, int* not_exact) {
-  int bad = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
-       i += (int64_t)gridDim.x * blockDim.x)
-    bad |= (__float_as_uint(x[i]) & 0x1FFFu) != 0;
-  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(not_exact, 1);
-}
-
 }  // namespace tc
 }  // namespace graph
 }  // namespace song

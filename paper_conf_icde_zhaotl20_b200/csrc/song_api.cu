@@ -103,6 +103,10 @@ __global__ void normalize_rows_kernel(float* data, int64_t n, int dpad) {
   }
 }
 
+int dpad_of(int dim, int metric) {
+  return (metric == SONG_HAMMING && (dim == 1 || dim == 2)) ? dim : (dim + 3) & ~3;
+}
+
 int alloc_index(song_index* ix, int64_t n, int32_t dim, int32_t degree, song_metric metric) {
   CUDA_TRY(cudaGetDevice(&ix->device));
   CUDA_TRY(cudaDeviceGetAttribute(&ix->num_sms, cudaDevAttrMultiProcessorCount, ix->device));
@@ -110,7 +114,7 @@ int alloc_index(song_index* ix, int64_t n, int32_t dim, int32_t degree, song_met
   ix->dim = dim;
   // float rows: 16 B multiples; codes: 1, 2 or a multiple of 4 words, so
   // h = 32 / 64 take exactly h / 8 bytes per point (Table IV)
-  ix->dpad = (metric == SONG_HAMMING && (dim == 1 || dim == 2)) ? dim : (dim + 3) & ~3;
+  ix->dpad = dpad_of(dim, (int)metric);
   ix->degree = degree;
   ix->metric = (int)metric;
   CUDA_TRY(cudaMalloc(&ix->d_data, (size_t)n * ix->dpad * sizeof(float)));
@@ -141,6 +145,7 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_qbin);
   cudaFree(ix->d_qcodes);
   if (ix->stream) cudaStreamDestroy(ix->stream);
+  if (ix->last_done) cudaEventDestroy(ix->last_done);
   delete ix;
 }
 
@@ -177,6 +182,7 @@ struct Shape {
   int warp_bytes;
   int qr;  // register queue width (L <= 32*qr), 0 = shared-memory queues
   int nch;
+  int warps;  // warps per CTA
 };
 
 // slots of the shared-memory visited hash: >= F (2L + 32), the live-key bound
@@ -229,11 +235,30 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
                  (s.qr == 0 ? 3 * L * 8 + 8 : 0) + tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
+  // CTA size (1 warp = 1 query): 4 warps unless shared memory is the limit
+  s.warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
+  while (s.warps > 1 && (size_t)s.warp_bytes * s.warps > 200 * 1024) s.warps >>= 1;
+  if (p->warps_per_block <= 0 && s.warp_bytes > 16 * 1024) {
+    // shared-memory-bound queue lengths: the CTA size that keeps the most warps
+    // resident (227 KB per SM; e.g. 73 KB per warp at L = 1536: 1-warp CTAs
+    // hold 3 warps per SM where 2-warp CTAs hold 2)
+    const size_t sm = 227 * 1024;
+    int best = 0;
+    for (int w = 4; w >= 1; w >>= 1) {
+      const size_t cta = (size_t)s.warp_bytes * w + 1024;  // + the per-CTA reservation
+      const int res = cta <= sm ? (int)(sm / cta) * w : 0;
+      if (res > best) {
+        best = res;
+        s.warps = w;
+      }
+    }
+  }
   return s;
 }
 
 
-int check_params(const song_index* ix, const song_search_params* p) {
+// the checks that need no index (song_search_plan_get and every search)
+int check_params_common(const song_search_params* p, int metric) {
   if (p->K < 1) return fail(SONG_EINVAL, "K must be >= 1");
   if (p->queue_len < p->K) return fail(SONG_EINVAL, "queue_len %d < K %d", p->queue_len, p->K);
   if (p->queue_len > SONG_MAX_QUEUE_LEN)
@@ -242,7 +267,6 @@ int check_params(const song_index* ix, const song_search_params* p) {
     return fail(SONG_EINVAL, "unknown visited kind %d", p->visited);
   if (p->table_log2 < 0 || p->table_log2 > 24)
     return fail(SONG_EUNSUPPORTED, "table_log2 %d outside [0, 24]", p->table_log2);
-  if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
   if (p->bloom_log2_bits < 0 || p->bloom_log2_bits > 24)
     return fail(SONG_EUNSUPPORTED, "bloom_log2_bits %d outside [0, 24]", p->bloom_log2_bits);
   if (p->warps_per_block < 0 || p->warps_per_block > SONG_LB_THREADS / 32)
@@ -262,8 +286,52 @@ int check_params(const song_index* ix, const song_search_params* p) {
   if (p->steps > SONG_MAX_STEPS)
     return fail(SONG_EUNSUPPORTED, "steps %d > %d", p->steps, SONG_MAX_STEPS);
   if (p->steps > 1 && ((p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM) ||
-                       ix->metric == SONG_HAMMING))
+                       metric == SONG_HAMMING))
     return fail(SONG_EUNSUPPORTED, "multi-step probing needs visited HASH or BLOOM on a float index");
+  if (metric == SONG_HAMMING && p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM)
+    return fail(SONG_EUNSUPPORTED, "Hamming indexes support the hash and Bloom visited sets");
+  if ((p->visited == SONG_VISITED_HASH_GLOBAL || p->visited == SONG_VISITED_HASH_GLOBAL_SEL) &&
+      p->table_log2 > 0 && (1 << (p->table_log2 - 1)) < SONG_MAX_DEGREE + 1)
+    // one iteration inserts up to 32 ids after a load check at 1/2: a smaller
+    // table could fill up inside an iteration and its probes would never end
+    return fail(SONG_EUNSUPPORTED, "table_log2 %d: the global visited table needs >= 2^7 slots",
+                p->table_log2);
+  return SONG_OK;
+}
+
+int check_params(const song_index* ix, const song_search_params* p) {
+  int rc = check_params_common(p, ix->metric);
+  if (rc) return rc;
+  if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
+  return SONG_OK;
+}
+
+// searches of one index share d_ticket / d_status and the order / query-code
+// scratch: a search on another stream waits for the previous one (song.h,
+// Concurrency)
+int order_after_last(song_index* ix, cudaStream_t st) {
+  if (st != ix->last_stream && ix->last_done) CUDA_TRY(cudaStreamWaitEvent(st, ix->last_done, 0));
+  ix->last_stream = st;
+  return SONG_OK;
+}
+
+// index-free part of a search's plan: the visited kind, the data-structure
+// sizes and the launch shape
+int vk_of(const song_search_params* p) {
+  switch (p->visited) {
+    case SONG_VISITED_BLOOM: return song::VK_BLOOM;
+    case SONG_VISITED_HASH_GLOBAL:
+    case SONG_VISITED_HASH_GLOBAL_SEL: return song::VK_GHASH;
+    case SONG_VISITED_CUCKOO: return song::VK_CUCKOO;
+    default: return song::VK_HASH;
+  }
+}
+
+int plan_shape(const song_search_params* p, int dpad, int metric, Shape* out) {
+  *out = search_shape(p->queue_len, vk_of(p), p, dpad, metric == SONG_HAMMING);
+  if ((size_t)out->warp_bytes * out->warps > 227 * 1024)
+    return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
+                p->queue_len, out->warp_bytes);
   return SONG_OK;
 }
 
@@ -336,27 +404,14 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);
   a.id_offset = p->id_offset;
   a.steps = p->steps > 1 ? p->steps : 1;
-  int warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
-  while (warps > 1 && (size_t)sh.warp_bytes * warps > 200 * 1024) warps >>= 1;
-  if (p->warps_per_block <= 0 && sh.warp_bytes > 16 * 1024) {
-    // shared-memory-bound queue lengths: the CTA size that keeps the most warps
-    // resident (227 KB per SM; e.g. 73 KB per warp at L = 1536: 1-warp CTAs
-    // hold 3 warps per SM where 2-warp CTAs hold 2)
-    const size_t sm = 227 * 1024;
-    int best = 0;
-    for (int w = 4; w >= 1; w >>= 1) {
-      const size_t cta = (size_t)sh.warp_bytes * w + 1024;  // + the per-CTA reservation
-      const int res = cta <= sm ? (int)(sm / cta) * w : 0;
-      if (res > best) {
-        best = res;
-        warps = w;
-      }
-    }
-  }
+  const int warps = sh.warps;
   if ((size_t)sh.warp_bytes * warps > 227 * 1024)
     return fail(SONG_EUNSUPPORTED, "queue_len %d needs %d B of shared memory per warp",
                 p->queue_len, sh.warp_bytes);
-  ix->last_stream = st;
+  // searches of one index share d_ticket / d_status / the order scratch: a
+  // search on another stream waits for the previous one (song.h, Concurrency)
+  int orc = order_after_last(ix, st);
+  if (orc) return orc;
   // ticket order (song_search_params.schedule): outlier-first needs the centroid
   // (float indexes) and pays when the batch outnumbers the resident warps
   const bool outlier_first =
@@ -369,12 +424,17 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
     a.order = ix->d_order;
   }
   const int m = ix->metric, qr = sh.qr, bps = p->blocks_per_sm, sms = ix->num_sms;
+  int rc;
   switch (sh.nch) {
-    case 1: return launch_m<1>(ix, a, m, vk, qr, warps, bps, sms, st);
-    case 2: return launch_m<2>(ix, a, m, vk, qr, warps, bps, sms, st);
-    case 4: return launch_m<4>(ix, a, m, vk, qr, warps, bps, sms, st);
-    default: return launch_m<8>(ix, a, m, vk, qr, warps, bps, sms, st);
+    case 1: rc = launch_m<1>(ix, a, m, vk, qr, warps, bps, sms, st); break;
+    case 2: rc = launch_m<2>(ix, a, m, vk, qr, warps, bps, sms, st); break;
+    case 4: rc = launch_m<4>(ix, a, m, vk, qr, warps, bps, sms, st); break;
+    default: rc = launch_m<8>(ix, a, m, vk, qr, warps, bps, sms, st); break;
   }
+  if (rc) return rc;
+  if (!ix->last_done) CUDA_TRY(cudaEventCreateWithFlags(&ix->last_done, cudaEventDisableTiming));
+  CUDA_TRY(cudaEventRecord(ix->last_done, st));
+  return SONG_OK;
 }
 
 int finish_create(song_index* ix, cudaStream_t st) {
@@ -661,6 +721,31 @@ int song_index_create_rp(const float* vectors, int64_t n, int32_t dim, const flo
 }
 
 
+int song_search_plan_get(const song_search_params* p, int32_t dim, int32_t metric,
+                         song_search_plan* out) {
+  if (!p || !out) return fail(SONG_EINVAL, "NULL argument");
+  std::memset(out, 0, sizeof *out);
+  if (dim < 1) return fail(SONG_EINVAL, "dim must be >= 1");
+  if (metric < SONG_L2 || metric > SONG_HAMMING) return fail(SONG_EINVAL, "metric %d", metric);
+  if (metric != SONG_HAMMING && dim > SONG_MAX_DIM)
+    return fail(SONG_EUNSUPPORTED, "dim %d > %d", dim, SONG_MAX_DIM);
+  if (metric == SONG_HAMMING && dim * 32 > SONG_MAX_CODE_BITS)
+    return fail(SONG_EUNSUPPORTED, "%d code words > %d bits", dim, SONG_MAX_CODE_BITS);
+  int rc = check_params_common(p, metric);
+  if (rc) return rc;
+  Shape sh;
+  rc = plan_shape(p, dpad_of(dim, metric), metric, &sh);
+  if (rc) return rc;
+  const int vk = vk_of(p);
+  out->visited_log2 = sh.table_log2;
+  out->visited_cap = vk != song::VK_HASH ? 0 : sh.lazy ? sh.rebuild_at : -1;
+  out->queue_regs = sh.qr;
+  out->row_chunks = sh.nch;
+  out->smem_per_warp = sh.warp_bytes;
+  out->warps_per_block = sh.warps;
+  return SONG_OK;
+}
+
 void song_default_params(song_search_params* p, int32_t K, int32_t queue_len) {
   if (!p) return;
   std::memset(p, 0, sizeof *p);
@@ -784,6 +869,8 @@ int song_search_ex(song_index* ix, const song_search_params* p, const float* que
   if (ix->metric == SONG_HAMMING) {
     if (!ix->d_R)
       return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
+    rc = order_after_last(ix, (cudaStream_t)stream);
+    if (rc) return rc;
     rc = encode_queries(ix, queries, nq, (cudaStream_t)stream);
     if (rc) return rc;
     queries = reinterpret_cast<const float*>(ix->d_qcodes);
@@ -854,6 +941,8 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
     ix->cap_out = obytes;
   }
   cudaStream_t st = ix->stream;
+  rc = order_after_last(ix, st);
+  if (rc) return rc;
   CUDA_TRY(cudaMemcpyAsync(ix->d_q, queries, qbytes, cudaMemcpyHostToDevice, st));
   const float* dq = ix->d_q;
   if (ix->metric == SONG_HAMMING) {

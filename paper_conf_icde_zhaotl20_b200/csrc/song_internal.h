@@ -25,6 +25,7 @@ struct song_index {
   uint64_t gen_next = 1;               // next generation base for d_gtab
   cudaStream_t stream = nullptr;       // owned; used by song_search
   cudaStream_t last_stream = nullptr;  // stream of the last search
+  cudaEvent_t last_done = nullptr;     // recorded after the last search's kernels
   // scratch for the host-buffer entry point
   float* d_q = nullptr;
   int32_t* d_ids = nullptr;

@@ -33,7 +33,8 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
-            "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward"]
+            "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward",
+            "song_search_plan_get"]
 
 
 class SongError(RuntimeError):
@@ -61,6 +62,13 @@ class IndexInfo(ctypes.Structure):
                 ("vector_bytes", ctypes.c_int64), ("graph_bytes", ctypes.c_int64),
                 ("device", ctypes.c_int32), ("num_sms", ctypes.c_int32),
                 ("code_bits", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+
+
+class SearchPlan(ctypes.Structure):
+    _fields_ = [("visited_log2", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
+                ("queue_regs", ctypes.c_int32), ("row_chunks", ctypes.c_int32),
+                ("smem_per_warp", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 2)]
 
 
 _lib = None
@@ -93,6 +101,8 @@ def lib():
         L.song_build_graph.argtypes = [P, i64, i32, i32, i32, P, P]
         L.song_build_graph_batched.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, P, P]
         L.song_build_graph_from_forward.argtypes = [P, i64, i32, i32, i32, P, P, P, P]
+        L.song_search_plan_get.argtypes = [ctypes.POINTER(SearchParams), i32, i32,
+                                           ctypes.POINTER(SearchPlan)]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -102,7 +112,7 @@ def lib():
                      "song_index_last_status", "song_merge_topk", "song_rp_encode",
                      "song_index_create_codes", "song_index_create_rp",
                      "song_search_codes_ex", "song_build_graph", "song_build_graph_batched",
-                     "song_build_graph_from_forward"):
+                     "song_build_graph_from_forward", "song_search_plan_get"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -377,14 +387,21 @@ def build_graph_from_forward(vectors, fwd_ids, fwd_dists, metric: str = "l2"):
     return adj
 
 
-def default_visited_cap(L: int) -> int:
-    """The default lazy-deletion capacity C of include/song.h (visited_cap = 0)."""
-    big = L > 128
-    need = (2 if big else 4 if L > 64 else 8) * (2 * L + 32)
-    slots = 1
-    while slots < need:
-        slots <<= 1
-    return 3 * slots // 4 if big else 5 * slots // 8
+def plan(params: "Params", dim: int, metric: str = "l2") -> SearchPlan:
+    """song_search_plan_get: the resolved sizes and launch shape of a search
+    (host-only, no GPU needed).  ``dim`` is the index dimension (code words
+    for "hamming")."""
+    out = SearchPlan()
+    cp = params.to_c()
+    _check(lib().song_search_plan_get(ctypes.byref(cp), int(dim), METRICS[metric],
+                                      ctypes.byref(out)))
+    return out
+
+
+def default_visited_cap(L: int, dim: int = 128, metric: str = "l2", K: int = 1) -> int:
+    """The lazy-deletion capacity C the library uses for visited_cap = 0
+    (read from song_search_plan_get, the single source of the default)."""
+    return int(plan(Params(K=min(K, L), queue_len=L), dim, metric).visited_cap)
 
 
 def rp_encode(vectors, R):

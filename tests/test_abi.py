@@ -65,6 +65,7 @@ def test_params_struct_layout_matches_header(tmp_path):
         'int main(void){printf("%zu %zu %zu %zu %zu\\n", sizeof(song_search_params),'
         ' sizeof(song_index_info), offsetof(song_index_info, vector_bytes),'
         ' offsetof(song_index_info, code_bits), offsetof(song_search_params, table_log2));'
+        'printf("%zu %zu\\n", sizeof(song_search_plan), offsetof(song_search_plan, warps_per_block));'
         'return 0;}\n')
     exe = tmp_path / "layout"
     subprocess.check_call(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(src),
@@ -72,7 +73,8 @@ def test_params_struct_layout_matches_header(tmp_path):
     c = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
     assert c == [ctypes.sizeof(song.SearchParams), ctypes.sizeof(song.IndexInfo),
                  song.IndexInfo.vector_bytes.offset, song.IndexInfo.code_bits.offset,
-                 song.SearchParams.table_log2.offset]
+                 song.SearchParams.table_log2.offset, ctypes.sizeof(song.SearchPlan),
+                 song.SearchPlan.warps_per_block.offset]
 
 
 def test_product_package_does_not_import_oracle():
@@ -110,3 +112,35 @@ def test_rp_argument_errors_need_no_gpu():
     R = np.zeros((64, 8), np.float32)
     R[0, 0] = np.nan
     assert lib.song_index_create_rp(P(v), 4, 8, P(R), 64, P(adj), 2, ctypes.byref(out)) == -1
+
+
+@pytest.mark.parametrize("L", [1, 10, 28, 32, 48, 64, 100, 128, 144, 512, 1280, 2048])
+def test_plan_lazy_capacity_bounds(L):
+    """song_search_plan_get (host-only) resolves the lazy-deletion capacity C
+    of reading R14 inside its stated bounds: C >= 2L + 32 (the live bound
+    |q| + |topk| + one iteration's candidates) and C <= 3/4 of the table."""
+    from paper_conf_icde_zhaotl20_b200 import song
+    p = song.plan(song.Params(K=1, queue_len=L), 128)
+    slots = 1 << p.visited_log2
+    assert 2 * L + 32 <= p.visited_cap <= 3 * slots // 4
+    assert p.queue_regs == (1 if L <= 32 else 2 if L <= 64 else 4 if L <= 128 else 0)
+    assert p.smem_per_warp * p.warps_per_block <= 227 * 1024
+    # eager deletion and multi-step probing report -1; other kinds 0
+    assert song.plan(song.Params(K=1, queue_len=L, visited_cap=-1), 128).visited_cap == -1
+    assert song.plan(song.Params(K=1, queue_len=L, steps=2), 128).visited_cap == -1
+    assert song.plan(song.Params(K=1, queue_len=L, visited="bloom"), 128).visited_cap == 0
+
+
+def test_plan_errors_need_no_gpu():
+    from paper_conf_icde_zhaotl20_b200 import song
+    with pytest.raises(song.SongError) as e:  # K > queue_len
+        song.plan(song.Params(K=20, queue_len=10), 128)
+    assert e.value.code == -1
+    with pytest.raises(song.SongError) as e:  # a global table that one iteration could fill
+        song.plan(song.Params(K=1, queue_len=10, visited="hashtable", table_log2=6), 128)
+    assert e.value.code == -4
+    song.plan(song.Params(K=1, queue_len=10, visited="hashtable", table_log2=7), 128)
+    with pytest.raises(song.SongError):  # Cuckoo on codes
+        song.plan(song.Params(K=1, queue_len=10, visited="cuckoo"), 4, "hamming")
+    with pytest.raises(song.SongError):
+        song.plan(song.Params(K=1, queue_len=10), 2048)

@@ -40,3 +40,44 @@ def test_graph_choice_and_builder_params_per_config():
         b = bench.build_params(CONFIGS[name])
         assert b == bench.BUILD
         assert b["queue_len"] == 128 and b["batch_shift"] == 2 and b["prefix"] == 1 << 16
+
+
+def test_gpus_flag_launches_ranks_gloo():
+    """`bench.py --gpus 2` without a torchrun environment re-launches itself
+    under torch.distributed.run with 2 ranks (CPU: gloo); rank 0 reports the
+    world it saw."""
+    import json
+    import subprocess
+    env = dict(os.environ)
+    env.pop("WORLD_SIZE", None)
+    env["SONG_BENCH_BACKEND"] = "gloo"
+    env["CUDA_VISIBLE_DEVICES"] = ""
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2",
+                          "--launch-check"], capture_output=True, text=True, env=env, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    assert lines[0]["n_gpus"] == 2 and lines[0]["backend"] == "gloo"
+    assert lines[0]["rank_sum"] == 3.0  # ranks 0 and 1 both joined
+
+
+def test_parity_gate_bars():
+    import numpy as np
+    gi = np.arange(2000).reshape(200, 10).astype(np.int32)
+    gd = np.linspace(1, 2, 2000).reshape(200, 10).astype(np.float32)
+    gc = np.ones((200, 2), np.int64)
+    truth = gi.copy()
+    ok = bench.parity_gate(gi, gd, gc, gi.copy(), gd.copy(), gc.copy(), truth, exact=True)
+    assert ok["ok"] and ok["ids_equal"] == 1.0
+    # one query of 200 differs: 0.995 passes the float bar, never the integer one
+    oi = gi.copy()
+    oi[0, 9] = 99999
+    f = bench.parity_gate(gi, gd, gc, oi, gd.copy(), gc.copy(), truth, exact=False)
+    assert f["ok"] and f["ids_equal"] == 0.995
+    assert not bench.parity_gate(gi, gd, gc, oi, gd.copy(), gc.copy(), truth, exact=True)["ok"]
+    oi[1, 9] = 99999  # two of 200: below 0.995
+    assert not bench.parity_gate(gi, gd, gc, oi, gd.copy(), gc.copy(), truth, exact=False)["ok"]
+    # a distance off by more than rtol 1e-5 fails
+    od = gd.copy()
+    od[5, 3] *= 1.001
+    assert not bench.parity_gate(gi, gd, gc, gi.copy(), od, gc.copy(), truth, exact=False)["ok"]

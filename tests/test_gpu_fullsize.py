@@ -94,7 +94,7 @@ def test_full_size_sampled_parity(name, K, sample):
         assert_exact(g, o)
     else:
         scale = float(np.abs(o[1][np.isfinite(o[1])]).max())
-        assert_close(g, o, truth[pick], id_frac=0.99 if cfg.metric == "cosine" else 0.995,
+        assert_close(g, o, truth[pick], id_frac=0.995,
                      scale=scale)
     assert (np.diff(gd, axis=1) >= 0).all()
     assert ((gi >= 0) & (gi < cfg.n)).all()

@@ -38,7 +38,7 @@ def test_toy():
 def test_integer_random_bit_exact(n, dim, D, path, monkeypatch):
     """ragged n (tile tails: 64-row SIMT tiles, 128-row tensor-core tiles),
     ragged dims (k tails), many exact ties; both forward-list paths (the
-    tensor-core path is exact on these tf32-representable integers)."""
+    tensor-core path is exact on these small integers: dim * max^2 < 2^24)."""
     if path != "auto":
         monkeypatch.setenv("SONG_GRAPH_PATH", path)
     rng = np.random.default_rng(n + dim + D)
@@ -178,3 +178,54 @@ def test_from_forward_bit_exact():
     np.testing.assert_array_equal(got.cpu().numpy(), want)
     np.testing.assert_array_equal(oracle.build_graph_from_forward(x, *oracle.forward_lists(x, 16)),
                                   oracle.build_graph(x, 16))
+
+
+def test_from_forward_knn_lists_bit_exact():
+    """Unrestricted kNN lists (each row's D nearest of ALL rows, itself
+    included at distance 0, mutual neighbours in both F and B): C(v) is taken
+    as a set — no self loop, no repeated id — on the GPU as in the oracle."""
+    x = og._int_data(1500, 16, 31)
+    D = 12
+    xn = x.astype(np.float64)
+    d = ((xn[:, None, :] - xn[None, :, :]) ** 2).sum(-1)
+    order = np.lexsort((np.broadcast_to(np.arange(len(x)), d.shape), d), axis=1)[:, :D]
+    fi = order.astype(np.int32)
+    fd = np.take_along_axis(d, order, 1).astype(np.float32)
+    want = oracle.build_graph_from_forward(x, fi, fd, nthreads=8)
+    s = song()
+    got = s.build_graph_from_forward(torch.as_tensor(x, device="cuda"),
+                                     torch.as_tensor(fi, device="cuda"),
+                                     torch.as_tensor(fd, device="cuda")).cpu().numpy()
+    np.testing.assert_array_equal(got, want)
+    for v, row in enumerate(got):
+        r = [int(j) for j in row if j >= 0]
+        assert v not in r and len(set(r)) == len(r)
+
+
+def test_builders_reject_bad_input():
+    s = song()
+    x = torch.randn(3000, 16, device="cuda")
+    x[2999, 3] = float("nan")  # the last row: outside any exact prefix
+    for build in (lambda: s.build_graph(x, 8),
+                  lambda: s.build_graph_batched(x, 8, prefix=100, queue_len=32),
+                  lambda: s.build_graph_batched(x, 8, prefix=5000, queue_len=32)):
+        with pytest.raises(s.SongError) as e:
+            build()
+        assert e.value.code == -1
+    x[2999, 3] = 0.0
+    fi = torch.zeros((3000, 8), dtype=torch.int32, device="cuda")
+    fd = torch.zeros((3000, 8), device="cuda")
+    fi[5, 2] = 3000  # outside [-1, n)
+    with pytest.raises(s.SongError) as e:
+        s.build_graph_from_forward(x, fi, fd)
+    assert e.value.code == -1
+
+
+def test_tensor_core_path_only_when_exact(monkeypatch):
+    """Non-integer data never takes the tensor-core Gram by default: the auto
+    path gives the FFMA path's graph bit for bit."""
+    rng = np.random.default_rng(9)
+    x = (rng.integers(0, 200, (1500, 64)) / 8.0).astype(np.float32)  # tf32-representable, not integer
+    auto = gbuild(x, 16)
+    monkeypatch.setenv("SONG_GRAPH_PATH", "simt")
+    np.testing.assert_array_equal(auto, gbuild(x, 16))

@@ -190,7 +190,7 @@ def main():
                 import oracle
                 pick = np.arange(0, a.nq, max(1, a.nq // a.parity_sample))[:a.parity_sample]
                 gi, gd, gc = (t.cpu().numpy() for t in idx.search(q, params=p, counters=True))
-                cap = int(__import__("paper_conf_icde_zhaotl20_b200.song", fromlist=["x"]).default_visited_cap(L_op))
+                cap = int(__import__("paper_conf_icde_zhaotl20_b200.song", fromlist=["x"]).default_visited_cap(L_op, cfg.dim, cfg.metric))
                 t1 = time.time()
                 oi, od, oc, _ = oracle.search(x.cpu().numpy(), adj_host, q.cpu().numpy()[pick], 10,
                                               L_op, flags=oracle.OPTIMIZED_LAZY, lazy_cap=cap,
