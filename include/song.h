@@ -107,7 +107,8 @@ typedef struct song_search_params {
                               reading R14).  0 = lazy deletion with the default capacity
                               C = 5S/8 for queue_len <= 128, 3S/4 above, where S =
                               2^ceil(log2(F (2L + 32))) table slots, F = 8 (L <= 64), 4 (L <= 128) or
-                              2; > 0 = lazy with C = visited_cap (2L + 32 <= C <= 3S/4,
+                              4/3 (song_search_plan_get reports the C in effect); > 0 =
+                              lazy with C = visited_cap (2L + 32 <= C <= 3S/4,
                               else SONG_EINVAL); -1 = eager deletion (every evicted vertex
                               erased at once, the paper's literal schedule).  Lazy: the
                               erasures are applied together (visited := ids(q) ∪
@@ -343,6 +344,18 @@ int song_build_graph_batched(const float* vectors, int64_t n, int32_t dim, song_
 int song_build_graph_from_forward(const float* vectors, int64_t n, int32_t dim,
                                   song_metric metric, int32_t degree, const int32_t* fwd_ids,
                                   const float* fwd_dists, int32_t* adjacency_out, void* stream);
+
+/* Instrumentation builds only (compiled with -DSONG_STAGE_TIMING, e.g.
+ * `python -m paper_conf_icde_zhaotl20_b200._build --define SONG_STAGE_TIMING
+ * --out libsong_stages.so`; never the product library): the SM cycles the
+ * searches of this index spent per stage since the last reset, summed over
+ * warps — cycles_out[0] pop / terminate / topk update (Alg. 1 lines 3-8),
+ * [1] candidate locating (§V), [2] bulk distance computation (§VI), [3]
+ * maintenance (§IV) — the in-kernel split of Fig. 10.
+ * Synchronises the index's last stream; reset != 0 zeroes the counters.
+ * Errors: SONG_EINVAL (NULL), SONG_EUNSUPPORTED (a build without the
+ * instrumentation; cycles_out is zeroed). */
+int song_stage_cycles(song_index* idx, uint64_t* cycles_out, int32_t reset);
 
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);

@@ -73,7 +73,27 @@ struct SearchArgs {
   uint64_t* gtab;  // VK_GHASH: [grid warps][2^table_log2] u64
   uint32_t gen0;   // VK_GHASH: generation base of this launch
   int warp_smem_bytes;
+  unsigned long long* stage_cycles;  // SONG_STAGE_TIMING builds: [4] SM cycles per stage
 };
+
+// SONG_STAGE_TIMING (a separate build, never the product library): lane 0 of
+// every warp reads clock64 at the stage boundaries of each iteration and adds
+// the cycles of pop/topk (a3), locate (a4), distance (a5) and maintenance
+// (a6) to stage_cycles[0..3] — the in-kernel split of Fig. 10
+#ifdef SONG_STAGE_TIMING
+#define SONG_ST_MARK(k)                      \
+  do {                                       \
+    if (lane == 0) {                         \
+      const long long t_ = clock64();        \
+      st_acc[k] += (unsigned long long)(t_ - st_t); \
+      st_t = t_;                             \
+    }                                        \
+  } while (0)
+#else
+#define SONG_ST_MARK(k) \
+  do {                  \
+  } while (0)
+#endif
 
 // ------------------------------------------------------------------- keys --
 __device__ __forceinline__ uint32_t f2ord(float f) {
@@ -523,6 +543,120 @@ __device__ __forceinline__ void merge_into(RegArr<QR>& q, uint64_t sdesc, int la
   }
 }
 
+// ------------------------------------------- shared-memory queues (> 128)
+// q and topk for queue_len > 128: sorted arrays in shared memory laid out as
+// a TIERED VECTOR — blocks of 64 keys, each block a small ring with its own
+// head, every block full except the last; lane c of the warp owns block c
+// (queue_len <= 2048 = 32 blocks) and keeps its head in a register.  An
+// insertion shifts keys inside ONE block and passes one key from each later
+// block to the next (all lanes at once: each later block rotates by one
+// slot); popping the minimum passes each block's first key down the same
+// way.  So both are a constant number of warp operations whatever the queue
+// length, where a flat sorted array moves O(L) keys per iteration (measured:
+// ring moves were 45 % of the instructions at L = 1280).
+struct Tier {
+  uint64_t* a;  // nblk * 64 slots
+  int size;     // logical elements (warp-uniform)
+  int hd;       // lane c: physical offset of block c's first element
+  __device__ __forceinline__ int nb() const { return (size + 63) >> 6; }
+  // element i (per lane, 0 <= i < 32 * 64); every lane of the warp must call
+  __device__ __forceinline__ uint64_t at(int i) const {
+    const int b = (i >> 6) & 31;
+    const int h = __shfl_sync(FULL, hd, b);
+    return a[(b << 6) | ((h + i) & 63)];
+  }
+  // number of elements < x, x per lane (uniform trip count)
+  __device__ __forceinline__ int rank_lane(uint64_t x) const {
+    const int n = size;
+    int lo = 0;
+    for (int step = 1 << (31 - __clz(n | 1)); step > 0; step >>= 1) {
+      const int j = lo + step - 1;
+      const uint64_t v = at(j < n ? j : 0);
+      lo = (j < n && v < x) ? lo + step : lo;
+    }
+    return lo;
+  }
+  // number of elements < x, x warp-uniform: the block (first keys, one per
+  // lane), then the position inside it (two keys per lane)
+  __device__ __forceinline__ int rank_warp(uint64_t x, int lane) const {
+    const int n = size, nbk = nb();
+    const uint64_t first = lane < nbk ? a[(lane << 6) | hd] : KEY_MAX;
+    const int k = __popc(__ballot_sync(FULL, first < x));  // blocks starting below x
+    if (k == 0) return 0;
+    const int b = k - 1;
+    const int cnt = min(64, n - (b << 6));
+    const int h = __shfl_sync(FULL, hd, b);
+    const uint64_t e0 = a[(b << 6) | ((h + lane) & 63)];
+    const uint64_t e1 = a[(b << 6) | ((h + lane + 32) & 63)];
+    return (b << 6) + __popc(__ballot_sync(FULL, lane < cnt && e0 < x)) +
+           __popc(__ballot_sync(FULL, lane + 32 < cnt && e1 < x));
+  }
+  // insert x (warp-uniform, not present) at its sorted position; the caller
+  // keeps size < 32 * 64 and within its block budget
+  __device__ __forceinline__ void insert(uint64_t x, int lane) {
+    const int n = size, nbk = nb();
+    const int pos = rank_warp(x, lane);
+    const int b = pos >> 6, o = pos & 63;
+    // reads: the last key of every full block >= b (it moves to the next block)
+    const bool full = ((lane + 1) << 6) <= n;
+    const uint64_t v = (lane >= b && lane < nbk && full) ? a[(lane << 6) | ((hd + 63) & 63)] : 0;
+    const uint64_t vin = __shfl_up_sync(FULL, v, 1);  // lane c: the key block c - 1 passes on
+    const int hb = __shfl_sync(FULL, hd, b & 31);
+    const int cnt = b < nbk ? min(64, n - (b << 6)) : 0;
+    const int s0 = (b << 6) | ((hb + lane) & 63), s1 = (b << 6) | ((hb + lane + 32) & 63);
+    const uint64_t e0 = a[s0], e1 = a[s1];
+    const uint64_t up0 = __shfl_up_sync(FULL, e0, 1), up1 = __shfl_up_sync(FULL, e1, 1);
+    const uint64_t e0_31 = __shfl_sync(FULL, e0, 31);
+    __syncwarp();
+    // block b: offsets k <= cnt (k < 64) take old[k] (k < o), x (k = o) or
+    // old[k - 1] (k > o); old[63] of a full block left as v above
+    if (b < nbk) {
+      const int k0 = lane, k1 = lane + 32;
+      const uint64_t p1 = lane == 0 ? e0_31 : up1;
+      if (k0 <= cnt) a[s0] = k0 < o ? e0 : (k0 == o ? x : up0);
+      if (k1 <= cnt && k1 < 64) a[s1] = k1 < o ? e1 : (k1 == o ? x : p1);
+    } else if (lane == b) {  // pos == n on a block boundary: a new block
+      hd = 0;
+      a[b << 6] = x;
+    }
+    // later blocks rotate by one slot and take the previous block's last key
+    if (lane > b && lane < nbk) {
+      hd = (hd + 63) & 63;
+      a[(lane << 6) | hd] = vin;
+    } else if (lane == nbk && b < nbk && (n & 63) == 0) {  // the last block overflowed
+      hd = 0;
+      a[lane << 6] = vin;
+    }
+    __syncwarp();
+    size = n + 1;
+  }
+  // remove the minimum (element 0)
+  __device__ __forceinline__ void pop_front(int lane) {
+    const int nbk = nb();
+    const uint64_t fo = lane < nbk ? a[(lane << 6) | hd] : 0;
+    const uint64_t fin = __shfl_down_sync(FULL, fo, 1);  // lane c: block c + 1's first key
+    __syncwarp();
+    if (lane < nbk) {
+      const int old = hd;
+      hd = (hd + 1) & 63;
+      if (lane < nbk - 1) a[(lane << 6) | old] = fin;  // the freed slot is block c's last
+    }
+    __syncwarp();
+    --size;
+  }
+  // topk insertion (§IV-C, Alg. 1 line 7): insert x (x < the maximum when
+  // full); returns the evicted maximum (old element L-1 when full) or KEY_MAX
+  __device__ __forceinline__ uint64_t push1(uint64_t x, int L, int lane) {
+    uint64_t ev = KEY_MAX;
+    if (size == L) {
+      ev = at(L - 1);
+      --size;
+    }
+    insert(x, lane);
+    return ev;
+  }
+};
+
 // ------------------------------------------------------- bulk distance --
 // §VI: distances of the nc candidates whose ids are in cid[0..nc) (shared).
 // Rows are staged R at a time in `stage` by cp.async (LDGSTS, 16 B per lane
@@ -901,14 +1035,17 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 // QR > 0: q / topk in registers (queue_len <= 32*QR); QR == 0: shared memory.
 // wide rows (NCH >= 4: d > 256 floats, or 512/1024-bit codes) hold 4-8 float4
 // of query per lane: give them 128 registers (4 CTAs/SM) instead of spilling
-template <int NCH>
+// shared-memory queues (QR == 0) are held to <= 20 warps per SM by their
+// shared memory anyway: 5 CTAs give them 102 registers (the ring moves keep
+// 4 keys per lane in flight) instead of spilling at 80
+template <int NCH, int QR = 1>
 struct MinBlocks {
-  static constexpr int value = NCH >= 4 ? 4 : SONG_LB_BLOCKS;
+  static constexpr int value = NCH >= 4 ? 4 : (QR == 0 ? 5 : SONG_LB_BLOCKS);
 };
 // MS: multi-step probing (a.steps pops per iteration, <= MAX_STEPS; §V)
 constexpr int MAX_STEPS = 4;
 template <int NCH, int METRIC, int VK, int QR, bool MS = false>
-__global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
+__global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH>::R;
@@ -926,11 +1063,12 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
   int* cid = reinterpret_cast<int*>(base + stage_bytes + qsm_bytes + 16);
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + (MS ? 32 * MAX_STEPS : 32));  // 32 keys
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
-  uint64_t* qa = ev + 32;                                               // QR == 0 only
-  uint64_t* qb = qa + (QR == 0 ? L : 0);
-  uint64_t* tk = qb + (QR == 0 ? L : 0);
+  // QR == 0 only: q and topk as tiered vectors of ceil(L / 64) blocks
+  const int tslots = QR == 0 ? ((L + 63) >> 6) << 6 : 0;
+  uint64_t* qa = ev + 32;
+  uint64_t* tk = qa + tslots;
   int* table = reinterpret_cast<int*>(                                  // 16 B aligned
-      (reinterpret_cast<uintptr_t>(tk + (QR == 0 ? L : 0)) + 15) & ~uintptr_t(15));
+      (reinterpret_cast<uintptr_t>(tk + tslots) + 15) & ~uintptr_t(15));
   // 32-bit words of the shared-memory visited table
   const int twords = VK == VK_HASH    ? (1 << a.table_log2)
                      : VK == VK_BLOOM ? ((1 << a.table_log2) >> 5)
@@ -1063,10 +1201,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
     RegArr<QR == 0 ? 1 : QR> q, tk_r;
     q.clear();
     tk_r.clear();
+    Tier qg{qa, 0, 0}, tg{tk, 0, 0};  // QR == 0
     if (QR > 0) {
       if (lane == 0) q.v[0] = ke;
-    } else if (lane == 0) {
-      qa[0] = ke;
+    } else {
+      if (lane == 0) qa[0] = ke;
+      qg.size = 1;
+      __syncwarp();
     }
     int qsize = 1, tsize = 0;
     int n_dist = 1, n_exp = 0, iters = 0;
@@ -1075,6 +1216,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
     int adjv = (lane < a.degree) ? __ldg(a.adj + (int64_t)a.entry * a.degree + lane) : -1;
     __syncwarp();
 
+#ifdef SONG_STAGE_TIMING
+    unsigned long long st_acc[4] = {0, 0, 0, 0};
+    long long st_t = clock64();
+#endif
     while (qsize > 0) {
       if (iters >= a.max_iters) {
         capped = true;
@@ -1087,8 +1232,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         now = __shfl_sync(FULL, q.v[0], 0);
         tmax = tk_r.get(L - 1);  // KEY_MAX unless topk is full
       } else {
-        now = qa[0];
-        tmax = (tsize == L) ? tk[L - 1] : KEY_MAX;
+        now = qg.at(0);
+        tmax = (tsize == L) ? tg.at(L - 1) : KEY_MAX;
       }
       if (tmax < now) break;  // topk full and its max beats now (lines 4-5)
       uint64_t evicted = KEY_MAX;
@@ -1101,40 +1246,17 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
 #pragma unroll
           for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) in_topk |= __any_sync(FULL, tk_r.v[r] == now);
         } else {
-          for (int b0 = 0; b0 < tsize; b0 += 32)
-            in_topk |= __any_sync(FULL, b0 + lane < tsize && tk[b0 + lane] == now);
+          const int r = tg.rank_warp(now, lane);
+          const uint64_t at_r = tg.at(r < tsize ? r : 0);
+          in_topk = r < tsize && at_r == now;
         }
       }
-      // push x into the shared-memory topk (L > 128); returns the evicted key
-      auto smem_topk_push = [&](uint64_t x) -> uint64_t {
-        const uint64_t out = (tsize == L) ? tk[L - 1] : KEY_MAX;
-        int pos = 0;
-        for (int b0 = 0; b0 < tsize; b0 += 32) {
-          int i = b0 + lane;
-          pos += __popc(__ballot_sync(FULL, i < tsize && tk[i] < x));
-        }
-        const int newsize = min(tsize + 1, L);
-        for (int b0 = ((newsize - 1) >> 5) << 5; b0 >= ((pos >> 5) << 5); b0 -= 32) {
-          int i = b0 + lane;
-          uint64_t val = 0;
-          bool w = false;
-          if (i > pos && i < newsize) {
-            val = tk[i - 1];
-            w = true;
-          } else if (i == pos) {
-            val = x;
-            w = true;
-          }
-          __syncwarp();
-          if (w) tk[i] = val;
-        }
-        return out;
-      };
       if (QR > 0) {
         if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
         q.pop_front(lane);
-      } else if (!in_topk) {
-        evicted = smem_topk_push(now);
+      } else {
+        qg.pop_front(lane);
+        if (!in_topk) evicted = tg.push1(now, L, lane);
       }
       if (!in_topk) tsize = min(tsize + 1, L);
       if (DEL) v_erase_lane0(evicted);  // §IV-E: topk's evicted vertex
@@ -1145,15 +1267,16 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
       int popid = key_id(now);  // lane i < npop: id of the i-th popped vertex
       if constexpr (MS) {
         for (; npop < a.steps && npop < qsize; ++npop) {
-          const uint64_t nx = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : qa[npop];
-          const uint64_t tm = (QR > 0) ? tk_r.get(L - 1) : ((tsize == L) ? tk[L - 1] : KEY_MAX);
+          const uint64_t nx = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : qg.at(0);
+          const uint64_t tm = (QR > 0) ? tk_r.get(L - 1) : ((tsize == L) ? tg.at(L - 1) : KEY_MAX);
           if (tm < nx) break;
           uint64_t ev1;
           if (QR > 0) {
             ev1 = tk_r.insert_one(nx, L, lane);
             q.pop_front(lane);
           } else {
-            ev1 = smem_topk_push(nx);
+            qg.pop_front(lane);
+            ev1 = tg.push1(nx, L, lane);
           }
           tsize = min(tsize + 1, L);
           if (DEL) v_erase_lane0(ev1);
@@ -1162,8 +1285,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         }
       }
       const int na = qsize - npop;  // q after the pops
-      const uint64_t* A = qa + npop;
 
+      SONG_ST_MARK(0);
       // ---- a4: candidate locating (§V)
       int v = adjv;
       bool keep = v >= 0;
@@ -1207,21 +1330,22 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
       // how it is split (the selection threshold is fixed within an iteration
       // and evictions = (q u new) minus its L smallest)
       int na_g = na;
-      const uint64_t* A_g = A;
       for (int g0 = 0;; g0 += 32) {
       const int nc = min(32, nc_all - g0);
       const int* cidg = cid + g0;
       const bool last_group = !MS || g0 + 32 >= nc_all;
 
+      SONG_ST_MARK(1);
       // ---- a5: bulk distance computation (§VI)
       const float dist =
           dist_of<NCH, METRIC>(a.data, a.dpad, cidg, nc, qv, qsm, stage, a.cosine, lane);
 
+      SONG_ST_MARK(2);
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cidg[lane] : -1;
       uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
       const uint64_t thr =
-          (a.sel && tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tk[L - 1]) : KEY_MAX;
+          (a.sel && tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tg.at(L - 1)) : KEY_MAX;
       // selected insertion: filtered only when worse than ALL of topk
       // (a key equal to topk's max can only arise from a filter false negative)
       const bool sel = (lane < nc) && key <= thr;
@@ -1230,7 +1354,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
       if (!sel) key = KEY_MAX;
       // prefetch the adjacency row of the next head = min(q head, best new key)
       if (last_group) {
-        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na_g > 0 ? A_g[0] : KEY_MAX);
+        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na_g > 0 ? qg.at(0) : KEY_MAX);
         uint64_t nxt = umin64(qhead, warp_min_key(key));
         if (nxt != KEY_MAX && lane < a.degree)
           adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
@@ -1266,10 +1390,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
                 hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
               }
             } else {
-              for (int i0 = 0; i0 < na_g; i0 += 32)
-                hs.insert(i0 + lane < na_g ? key_id(A_g[i0 + lane]) : 0, i0 + lane < na_g);
-              for (int i0 = 0; i0 < tsize; i0 += 32)
-                hs.insert(i0 + lane < tsize ? key_id(tk[i0 + lane]) : 0, i0 + lane < tsize);
+              for (int i0 = 0; i0 < na_g; i0 += 32) {
+                const uint64_t kq = qg.at(i0 + lane < na_g ? i0 + lane : 0);  // (all lanes)
+                hs.insert(key_id(kq), i0 + lane < na_g);
+              }
+              for (int i0 = 0; i0 < tsize; i0 += 32) {
+                const uint64_t kt = tg.at(i0 + lane < tsize ? i0 + lane : 0);
+                hs.insert(key_id(kt), i0 + lane < tsize);
+              }
             }
             used = na_g + tsize;
             __syncwarp();
@@ -1333,15 +1461,21 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
             cuckoo_erase_sorted_desc(ne);
           }
         }
-      } else {
+      } else {  // QR == 0: the q ring
         visit_selected();
         __syncwarp();
-        key = bitonic_sort32<false>(key, lane);
+        // compact the selected keys to lanes [0, ns) and sort only those
+        if (sel) keys32[__popc(smask & lt)] = key;
+        __syncwarp();
+        key = lane < ns ? keys32[lane] : KEY_MAX;
+        __syncwarp();
+        key = sort_prefix(key, ns, lane);
         int nsq = ns;  // selected keys that enter q
         if constexpr (VK == VK_CUCKOO) {
           // drop keys already in q (Cuckoo false negatives), re-compact
-          const int j = count_below(A_g, na_g, key);
-          const bool dup = lane < ns && j < na_g && A_g[j] == key;
+          const int j = qg.rank_lane(key);
+          const uint64_t at_j = qg.at(j < na_g ? j : 0);
+          const bool dup = lane < ns && j < na_g && at_j == key;
           const unsigned keepm = __ballot_sync(FULL, lane < ns && !dup);
           nsq = __popc(keepm);
           __syncwarp();
@@ -1350,42 +1484,57 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
           key = lane < nsq ? keys32[lane] : KEY_MAX;
           __syncwarp();
         }
-        keys32[lane] = key;
-        __syncwarp();
-        // merged position p >= L is evicted: ev[p - L] (< 32 of them) in key order
-        for (int i0 = 0; i0 < na_g; i0 += 32) {
-          const int i = i0 + lane;
-          const uint64_t x = i < na_g ? A_g[i] : KEY_MAX;
-          const int p = i + count_below(keys32, nsq, x);
-          if (i < na_g && p < L) qb[p] = x;
-          if (i < na_g && p >= L) ev[p - L] = x;
-          if constexpr (VK == VK_HASH) hs.erase(key_id(x), i < na_g && p >= L && !a.lazy);
+        if (nsq > 0) {
+          // insert the new keys in ascending order; a full q evicts its
+          // maximum first (§IV-C) — the evicted set is the largest
+          // (na + nsq - L) keys of q and the new ones, as a merge would give
+          int ne = 0;
+          uint64_t evk = KEY_MAX;  // lane e: the e-th evicted key
+          for (int j = 0; j < nsq; ++j) {
+            const uint64_t x = __shfl_sync(FULL, key, j);
+            if (qg.size == L) {
+              const uint64_t mx = qg.at(L - 1);
+              if (x > mx) {  // x and every later key are evicted at once
+                const uint64_t moved = __shfl_sync(FULL, key, (lane - ne + j) & 31);
+                if (lane >= ne && lane < ne + nsq - j) evk = moved;
+                ne += nsq - j;
+                break;
+              }
+              if (lane == ne) evk = mx;
+              ++ne;
+              qg.size = L - 1;
+            }
+            qg.insert(x, lane);
+          }
+          if (ne > 0) {
+            if constexpr (VK == VK_HASH) hs.erase(key_id(evk), lane < ne && !a.lazy);  // §IV-E
+            if constexpr (VK == VK_CUCKOO) {
+              // ascending, then erased from the largest down (reading R9)
+              const uint64_t srt = sort_prefix(lane < ne ? evk : KEY_MAX, ne, lane);
+              ev[lane] = srt;
+              __syncwarp();
+              cuckoo_erase_sorted_desc(ne);
+            }
+          }
         }
-        {
-          const int p = lane + count_below(A_g, na_g, key);
-          if (lane < nsq && p < L) qb[p] = key;
-          if (lane < nsq && p >= L) ev[p - L] = key;
-          if constexpr (VK == VK_HASH) hs.erase(key_id(key), lane < nsq && p >= L && !a.lazy);
-        }
-        __syncwarp();
-        if constexpr (VK == VK_CUCKOO) cuckoo_erase_sorted_desc(max(0, na_g + nsq - L));
-        qsize_new = min(na_g + nsq, L);
-        uint64_t* t = qa;
-        qa = qb;
-        qb = t;
+        qsize_new = qg.size;
       }
       qsize = qsize_new;
       __syncwarp();
       na_g = qsize;
-      A_g = qa;
       if (last_group) break;
       }  // candidate groups
+      SONG_ST_MARK(3);
       if (VK == VK_GHASH && used > (1 << (a.table_log2 - 1))) {  // keep load <= 1/2
         full = true;
         break;
       }
     }
 
+#ifdef SONG_STAGE_TIMING
+    if (lane == 0 && a.stage_cycles)
+      for (int k = 0; k < 4; ++k) atomicAdd(a.stage_cycles + k, st_acc[k]);
+#endif
     // ---- a7: output the first K of topk (Alg. 1 line 17)
     if (QR > 0) {
 #pragma unroll
@@ -1398,18 +1547,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH>::value)
         }
       }
     } else {
-      for (int i = lane; i < a.K; i += 32) {
-        if (i < tsize) {
-          uint64_t k = tk[i];
-          ids_o[i] = key_id(k) + a.id_offset;
-          dists_o[i] = ord2f((uint32_t)(k >> 32));
-        } else {
-          ids_o[i] = -1;
-          dists_o[i] = __int_as_float(0x7f800000);
+      for (int i0 = 0; i0 < a.K; i0 += 32) {
+        const int i = i0 + lane;
+        const uint64_t k = tg.at(i < tsize ? i : 0);  // (every lane calls: shuffles)
+        if (i < a.K) {
+          ids_o[i] = i < tsize ? key_id(k) + a.id_offset : -1;
+          dists_o[i] = i < tsize ? ord2f((uint32_t)(k >> 32)) : __int_as_float(0x7f800000);
         }
       }
-      qa = ev + 32;
-      qb = qa + L;
     }
     if (a.counters_out && lane == 0) {
       a.counters_out[2 * (int64_t)qi] = n_dist;

@@ -144,6 +144,7 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_order);
   cudaFree(ix->d_qbin);
   cudaFree(ix->d_qcodes);
+  cudaFree(ix->d_stage);
   if (ix->stream) cudaStreamDestroy(ix->stream);
   if (ix->last_done) cudaEventDestroy(ix->last_done);
   delete ix;
@@ -185,10 +186,21 @@ struct Shape {
   int warps;  // warps per CTA
 };
 
-// slots of the shared-memory visited hash: >= F (2L + 32), the live-key bound
+// slots of the shared-memory visited hash: >= F (2L + 32), the live-key bound;
+// shared-memory queues (L > 128) take F = 4/3 — the least table whose 3/4
+// still holds the bound (measured: at L = 1280 the 32 KB table of F = 2 held
+// 3 warps per SM, the 16 KB one holds 5)
+#ifndef SONG_HASH_BIG_NUM
+#define SONG_HASH_BIG_NUM 4
+#endif
+#ifndef SONG_HASH_BIG_DEN
+#define SONG_HASH_BIG_DEN 3
+#endif
 int hash_log2_slots(int L) {
-  const long long F = L > 128 ? 2 : L > 64 ? SONG_HASH_FACTOR_WIDE : SONG_HASH_FACTOR;
-  return next_pow2_log2(F * (2ll * L + 32));
+  const long long live = 2ll * L + 32;
+  if (L > 128) return next_pow2_log2((SONG_HASH_BIG_NUM * live + SONG_HASH_BIG_DEN - 1) / SONG_HASH_BIG_DEN);
+  const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE : SONG_HASH_FACTOR;
+  return next_pow2_log2(F * live);
 }
 
 Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
@@ -233,7 +245,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
   s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
-                 (s.qr == 0 ? 3 * L * 8 + 8 : 0) + tbytes;
+                 (s.qr == 0 ? 2 * (((L + 63) / 64) * 64) * 8 + 8 : 0) + tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   // CTA size (1 warp = 1 query): 4 warps unless shared memory is the limit
   s.warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
@@ -393,6 +405,14 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   }
   a.gtab = nullptr;
   a.gen0 = 0;
+  a.stage_cycles = nullptr;
+#ifdef SONG_STAGE_TIMING
+  if (!ix->d_stage) {
+    CUDA_TRY(cudaMalloc(&ix->d_stage, 4 * sizeof(unsigned long long)));
+    CUDA_TRY(cudaMemset(ix->d_stage, 0, 4 * sizeof(unsigned long long)));
+  }
+  a.stage_cycles = ix->d_stage;
+#endif
   if (ix->metric == SONG_HAMMING && vk != song::VK_HASH && vk != song::VK_BLOOM)
     return fail(SONG_EUNSUPPORTED, "Hamming indexes support the hash and Bloom visited sets");
   Shape sh = search_shape(p->queue_len, vk, p, ix->dpad, ix->metric == SONG_HAMMING);
@@ -973,6 +993,24 @@ int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int
       ids_in, dists_in, G, nq, Kin, K, ids_out, dists_out);
   CUDA_TRY(cudaGetLastError());
   return SONG_OK;
+}
+
+int song_stage_cycles(song_index* ix, uint64_t* cycles_out, int32_t reset) {
+  if (!ix || !cycles_out) return fail(SONG_EINVAL, "NULL argument");
+#ifdef SONG_STAGE_TIMING
+  CUDA_TRY(cudaStreamSynchronize(ix->last_stream));
+  if (!ix->d_stage) {
+    for (int k = 0; k < 4; ++k) cycles_out[k] = 0;
+    return SONG_OK;
+  }
+  CUDA_TRY(cudaMemcpy(cycles_out, ix->d_stage, 4 * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  if (reset) CUDA_TRY(cudaMemset(ix->d_stage, 0, 4 * sizeof(uint64_t)));
+  return SONG_OK;
+#else
+  (void)reset;
+  for (int k = 0; k < 4; ++k) cycles_out[k] = 0;
+  return fail(SONG_EUNSUPPORTED, "this libsong.so was built without SONG_STAGE_TIMING");
+#endif
 }
 
 const char* song_last_error(void) { return g_err.c_str(); }

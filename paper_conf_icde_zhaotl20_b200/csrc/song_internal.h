@@ -44,6 +44,7 @@ struct song_index {
   uint16_t* d_qbin = nullptr;          // [nq] bin of each query
   size_t cap_order = 0;
   int* h_status = nullptr;             // pinned: song_search's status read-back
+  unsigned long long* d_stage = nullptr;  // SONG_STAGE_TIMING builds: [4] cycles
 };
 
 namespace song {

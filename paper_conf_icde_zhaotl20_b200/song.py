@@ -34,7 +34,7 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
             "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward",
-            "song_search_plan_get"]
+            "song_search_plan_get", "song_stage_cycles"]
 
 
 class SongError(RuntimeError):
@@ -103,6 +103,7 @@ def lib():
         L.song_build_graph_from_forward.argtypes = [P, i64, i32, i32, i32, P, P, P, P]
         L.song_search_plan_get.argtypes = [ctypes.POINTER(SearchParams), i32, i32,
                                            ctypes.POINTER(SearchPlan)]
+        L.song_stage_cycles.argtypes = [P, P, i32]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -112,7 +113,8 @@ def lib():
                      "song_index_last_status", "song_merge_topk", "song_rp_encode",
                      "song_index_create_codes", "song_index_create_rp",
                      "song_search_codes_ex", "song_build_graph", "song_build_graph_batched",
-                     "song_build_graph_from_forward", "song_search_plan_get"):
+                     "song_build_graph_from_forward", "song_search_plan_get",
+                     "song_stage_cycles"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -304,6 +306,13 @@ class SongIndex:
             ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(dists.data_ptr()),
             ctypes.c_void_p(ctr.data_ptr() if ctr is not None else 0), _stream_ptr(q.device)))
         return (ids, dists, ctr) if counters else (ids, dists)
+
+    def stage_cycles(self, reset: bool = True):
+        """song_stage_cycles (SONG_STAGE_TIMING builds): SM cycles per stage
+        [pop/topk, locate, distance, maintenance] summed over warps."""
+        out = np.zeros(4, np.uint64)
+        _check(lib().song_stage_cycles(self._h, out.ctypes.data_as(ctypes.c_void_p), int(reset)))
+        return out
 
     def last_status(self):
         """Synchronise and raise SongError if a query was flagged."""
