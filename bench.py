@@ -93,6 +93,8 @@ def parse():
     ap.add_argument("--target-recall", type=float, default=0.95)
     ap.add_argument("--queue-len", type=int, default=0, help="skip the sweep")
     ap.add_argument("--visited", default="hash", choices=["hash", "bloom"])
+    ap.add_argument("--queue-kind", default="auto", choices=["auto", "separate", "union"],
+                    help="song_search_params.queue_kind (results never depend on it)")
     ap.add_argument("--warps-per-block", type=int, default=0)
     ap.add_argument("--blocks-per-sm", type=int, default=0)
     ap.add_argument("--visited-cap", type=int, default=0,
@@ -365,7 +367,7 @@ def run_song(args, ws, rank, local, log):
     def params(L):
         return song.Params(K=cfg.K, queue_len=L, visited=args.visited,
                            warps_per_block=args.warps_per_block, blocks_per_sm=args.blocks_per_sm,
-                           visited_cap=args.visited_cap)
+                           visited_cap=args.visited_cap, queue_kind=args.queue_kind)
 
     # ---- operating point: smallest grid queue_len with recall@10 >= target
     sweep = []
@@ -384,7 +386,8 @@ def run_song(args, ws, rank, local, log):
     ids, _ = idx.search(q0, params=params(L_op))
     rec = recall_t(ids, truth0)
     # the lazy-deletion capacity the library resolves (the oracle's lazy_cap)
-    cap = int(song.plan(params(L_op), cfg.dim, cfg.metric).visited_cap)
+    plan_op = song.plan(params(L_op), cfg.dim, cfg.metric)
+    cap, qkind = int(plan_op.visited_cap), int(plan_op.queue_kind)
     log(f"operating point L={L_op} recall={rec:.4f} sweep={sweep}")
     if args.sweep_only:
         return None
@@ -489,7 +492,7 @@ def run_song(args, ws, rank, local, log):
             "graph": graph_used, "n": cfg.n, "dim": d, "degree": deg, "nq_per_gpu": nq, "query_replicas": reps, "K": K, "queue_len": L_op,
             f"recall_at_{K}": round(rec, 4), "recall_sweep": sweep, "visited": args.visited,
             "visited_cap": args.visited_cap or "default (lazy deletion, reading R14)",
-            "visited_cap_resolved": cap,
+            "visited_cap_resolved": cap, "queue_kind": ["registers", "separate q, topk", "bounded union (R17)"][qkind],
             "l2": "flushed between timed steps (512 MiB write)",
             "parallelism": f"query-sharded dp{ws} (graph replicated per GPU)",
         },
@@ -575,7 +578,7 @@ def run_song(args, ws, rank, local, log):
         truth = truth0.cpu().numpy()
         if reps > 1:
             truth = np.tile(truth, (reps, 1))
-        base, parity = cpu_baseline(args, x, adj, q if rank == 0 else q0, truth, cfg, L_op, cap,
+        base, parity = cpu_baseline(args, x, adj, q, truth, cfg, L_op, (cap, qkind),
                                     ids_c, dists_c, ctr, log, timing=ws == 1 and not args.no_cpu_baseline)
         if base is not None:
             result["cpu_baseline"] = base
@@ -587,17 +590,19 @@ def run_song(args, ws, rank, local, log):
     return result
 
 
-def oracle_mode(L, cap, visited="hash"):
+def oracle_mode(L, cap, visited="hash", queue_kind=0):
     """The oracle mode of the GPU's search: selected insertion + lazy visited
     deletion (reading R14) with the capacity the library resolved for this
-    search (`cap` = song_search_plan_get's visited_cap; -1 = eager deletion);
+    search (`cap` = song_search_plan_get's visited_cap; -1 = eager deletion),
+    over the bounded union of reading R17 when the plan's queue_kind is 2;
     Bloom: the filter of reading A11."""
     import oracle
     if visited == "bloom":
         return dict(flags=oracle.OPTIMIZED_BLOOM, bloom_bits=oracle.default_bloom_bits(L))
+    uni = oracle.UNION if queue_kind == 2 else 0
     if cap == -1:
-        return dict(flags=oracle.OPTIMIZED)
-    return dict(flags=oracle.OPTIMIZED_LAZY, lazy_cap=cap)
+        return dict(flags=oracle.OPTIMIZED | uni)
+    return dict(flags=oracle.OPTIMIZED_LAZY | uni, lazy_cap=cap)
 
 
 # north_star parity bars (BASELINE.json): ids identical on >= 99.5 % of queries,
@@ -668,7 +673,7 @@ def cpu_baseline(args, x, adj, q, truth, cfg, L, cap, ids_c, dists_c, ctr, log, 
     import oracle
     cores = len(os.sched_getaffinity(0))
     xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()
-    mode = oracle_mode(L, cap, args.visited)
+    mode = oracle_mode(L, cap[0], args.visited, cap[1])
     t = time.perf_counter()
     oi, od, oc, _ = oracle.search(xn, an, qn, cfg.K, L, metric=oracle.METRICS[cfg.metric],
                                   nthreads=cores, **mode)
@@ -714,9 +719,11 @@ def emit_graph(args, log):
     dev = torch.device("cuda", 0)
     graph_used = default_graph(cfg) if args.graph == "auto" else args.graph
     x, q0, q, adj = build_workload(cfg, dev, 0, log, "", graph_used)
-    caps = {L: song.default_visited_cap(L, cfg.dim, cfg.metric, cfg.K) for L in grid_for(cfg.K)}
+    plans = {L: song.plan(song.Params(K=cfg.K, queue_len=L), cfg.dim, cfg.metric)
+             for L in grid_for(cfg.K)}
+    caps = [(L, p.visited_cap, p.queue_kind) for L, p in sorted(plans.items())]
     np.savez(args.emit_graph, adj=adj.cpu().numpy(), x_sum=float(x.double().sum()),
-             caps=np.array(sorted(caps.items()), dtype=np.int64), graph=graph_used)
+             caps=np.array(caps, dtype=np.int64), graph=graph_used)
 
 
 def reference_graph(args, cfg, log):
@@ -733,7 +740,7 @@ def reference_graph(args, cfg, log):
             cmd += [flag, str(BUILD[key])]
     subprocess.check_call(cmd)
     z = np.load(path)
-    caps = {int(L): int(c) for L, c in z["caps"]}
+    caps = {int(L): (int(c), int(k)) for L, c, k in z["caps"]}
     return z["adj"], float(z["x_sum"]), caps, str(z["graph"])
 
 
@@ -761,7 +768,7 @@ def run_reference(args, ws, rank, local, log):
     if not L_op:  # same operating-point rule as the song arm, on the same full batch
         for L in grid_for(cfg.K):
             ids, _, _, _ = oracle.search(xn, an, qn, cfg.K, L, metric=m, nthreads=cores,
-                                         **oracle_mode(L, caps[L]))
+                                         **oracle_mode(L, *caps[L]))
             r = oracle.recall(ids, truth)
             sweep.append((L, round(r, 4)))
             if r >= args.target_recall:
@@ -770,7 +777,7 @@ def run_reference(args, ws, rank, local, log):
     cap = caps.get(L_op)
     if cap is None:
         cap = caps[min(c for c in caps if c >= L_op)]
-    mode = oracle_mode(L_op, cap)
+    mode = oracle_mode(L_op, cap[0], "hash", cap[1])
     t = time.perf_counter()
     oracle.search(xn, an, qn[:64], cfg.K, L_op, metric=m, nthreads=cores, **mode)
     per_q = (time.perf_counter() - t) / 64
@@ -805,7 +812,8 @@ def run_reference(args, ws, rank, local, log):
         "cpu_baseline": {"value": round(value, 1), "unit": "queries/s", "cores": cores,
                          "kind": "oracle",
                          "sample": f"{S} queries per step (bounded), oracle hash-sel-del mode with "
-                                   f"lazy deletion (cap {cap}, the library's plan), as the GPU runs",
+                                   f"lazy deletion (cap {cap[0]}, queue kind {cap[1]}: the "
+                                   f"library's plan), as the GPU runs",
                          "single_thread": {"value": round(single[0], 1), "unit": "queries/s",
                                            "cores": 1,
                                            "sample": f"first {single[1]} queries x {single[2]} "

@@ -127,7 +127,25 @@ typedef struct song_search_params {
                               scheduling: far-out queries search longest),
                               in 4096 log-spaced key bins.  Codes indexes always use
                               batch order. */
+  int32_t queue_kind;      /* how q and topk are held (results never depend on it).
+                              SONG_QUEUE_AUTO (0, default): registers for queue_len <=
+                              128; above, with visited HASH and steps <= 1, the bounded
+                              union, else separate shared-memory q and topk.
+                              SONG_QUEUE_SEPARATE: q and topk as the paper keeps them
+                              (§IV-C), each bounded at L.  SONG_QUEUE_UNION (DESIGN.md
+                              reading R17): ONE list of the L best keys of q ∪ topk,
+                              each marked popped or not — the next pop is its first
+                              unpopped key, the search stops when none is left; the
+                              hash then holds <= L + 32 live ids (lazy capacity C in
+                              [L + 32, 3S/4], default 3S/4, S = 2^ceil(log2(8 (L + 32)
+                              / 3))) and a vertex dropped from the list is recomputed if
+                              met again (counters differ, results do not).  UNION needs
+                              visited HASH and steps <= 1 (else SONG_EUNSUPPORTED). */
 } song_search_params;
+
+#define SONG_QUEUE_AUTO 0
+#define SONG_QUEUE_SEPARATE 1
+#define SONG_QUEUE_UNION 2
 
 #define SONG_SCHEDULE_AUTO 0
 #define SONG_SCHEDULE_BATCH 1
@@ -166,7 +184,8 @@ typedef struct song_search_plan {
                               BLOOM: log2 bits m (reading A11); CUCKOO: log2 buckets of
                               4 fingerprints (reading R10) */
   int32_t visited_cap;     /* SONG_VISITED_HASH: the capacity C of lazy deletion in effect
-                              (reading R14; the oracle's lazy_cap), or -1 for eager
+                              (reading R14, or R17's when queue_kind is 2; the oracle's
+                              lazy_cap), or -1 for eager
                               deletion (visited_cap = -1 or steps > 1); 0 for the other
                               kinds */
   int32_t queue_regs;      /* q and topk held in registers, queue_regs u64 per lane
@@ -174,7 +193,9 @@ typedef struct song_search_plan {
   int32_t row_chunks;      /* 16 B chunks per lane of a staged row (NCH) */
   int32_t smem_per_warp;   /* shared-memory bytes per warp */
   int32_t warps_per_block; /* CTA size of the persistent grid (1 warp = 1 query) */
-  int32_t reserved[2];     /* 0 */
+  int32_t queue_kind;      /* 0 registers, 1 separate shared-memory q and topk, 2 the
+                              bounded union of reading R17 (song_search_params.queue_kind) */
+  int32_t reserved;        /* 0 */
 } song_search_plan;
 
 /* Errors: SONG_EINVAL (NULL, bad params as song_search_ex would report them,

@@ -44,6 +44,9 @@ OPTIMIZED_CUCKOO = BOUNDED_Q | SEL | DEL | CUCKOO  # "cuckoofilter" (Fig. 7)
 HASHTABLE = BOUNDED_Q                      # "hashtable" (Fig. 7): no sel, no del
 HASHTABLE_SEL = BOUNDED_Q | SEL            # "hashtable-sel" (Fig. 7)
 OPTIMIZED_LAZY = OPTIMIZED | LAZY          # hash-sel-del with lazy deletion (R14)
+UNION = 64  # q and topk as one bounded list of the L best discovered keys (reading R17)
+OPTIMIZED_UNION = OPTIMIZED | UNION
+OPTIMIZED_UNION_LAZY = OPTIMIZED_LAZY | UNION
 
 _TRACE_FN = ctypes.CFUNCTYPE(
     None, ctypes.c_void_p, ctypes.c_int64,

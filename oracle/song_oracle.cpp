@@ -105,6 +105,7 @@ enum Flags {
   ORACLE_BLOOM = 8,      // §IV-B: visited is a Bloom filter (no deletion)
   ORACLE_CUCKOO = 16,    // visited is a Cuckoo filter (supports deletion)
   ORACLE_LAZY = 32,      // with DEL: deletions deferred until visited reaches a capacity (R14)
+  ORACLE_UNION = 64,     // R17: q and topk kept as ONE bounded list (see search_one_union)
 };
 
 struct Key {
@@ -448,6 +449,117 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
   return status;
 }
 
+// Reading R17 — the bounded union.  q and topk of Algorithm 1 held as one
+// list W of the L smallest keys discovered (the vertices of q ∪ topk that can
+// still matter), each marked popped (in topk) or not (in q):
+//   1. W = {(d_e, e)} unpopped; visited = {e}; n_dist = 1.
+//   2. u = the smallest unpopped key of W; none -> stop (then every key of W
+//      is popped: topk is full and its max beats q's min, Alg. 1 lines 4-5,
+//      or q is empty).  Mark u popped (Alg. 1 lines 3, 7); n_exp += 1.
+//   3. Locate the unvisited neighbours of u (row order, first occurrence).
+//   4. Distances; n_dist += |cand|.
+//   5. Maintain: [sel] skip c when |W| = L and key(c) > max(W) (a key beaten
+//      by L discovered ones can never be popped nor returned); [lazy] if
+//      |visited| + selected > C first set visited := ids(W); insert the
+//      selected into visited and W (unpopped); while |W| > L drop max(W) and
+//      [del] erase it from visited.
+//   6. Return the first K popped keys of W (all of W is popped at the end).
+// Same popped sequence and result as Algorithm 1 (the popped key is q's min
+// whenever it lies in the best L of q ∪ topk; otherwise topk is full and
+// beats it — the stop rule), so the counters differ from the separate
+// structures only in n_dist: a vertex dropped from W is no longer visited
+// and is recomputed (then skipped by [sel]) if met again.
+int search_one_union(const Problem& P, const float* p, int32_t* ids_out, float* dists_out,
+                     int64_t* counters) {
+  const int L = P.L;
+  const bool sel = P.flags & ORACLE_SEL;
+  const bool lazy = (P.flags & ORACLE_LAZY) && (P.flags & ORACLE_DEL);
+  const bool del = (P.flags & ORACLE_DEL) && !lazy;
+  std::set<Key> W;
+  std::unordered_set<int32_t> popped;  // ids of W's popped keys
+  std::unordered_set<int32_t> visited;
+  int64_t n_dist = 0, n_exp = 0;
+  int status = 0;
+  const int32_t e = P.entry;
+  W.insert(Key{distance(p, P.data + (int64_t)e * P.dim, P.dim, P.metric), e});
+  visited.insert(e);
+  n_dist = 1;
+  std::vector<int32_t> cand;
+  int64_t it = 0;
+  while (true) {
+    Key u{0.f, -1};
+    for (const Key& k : W)
+      if (!popped.count(k.id)) {
+        u = k;
+        break;
+      }
+    if (u.id < 0) break;
+    if (it >= P.max_iters) {
+      status = 1;
+      break;
+    }
+    ++it;
+    popped.insert(u.id);
+    ++n_exp;
+    cand.clear();
+    const int32_t* row = P.adj + (int64_t)u.id * P.degree;
+    for (int j = 0; j < P.degree; ++j) {
+      const int32_t v = row[j];
+      if (v < 0 || visited.count(v)) continue;
+      if (std::find(cand.begin(), cand.end(), v) != cand.end()) continue;
+      cand.push_back(v);
+    }
+    std::vector<Key> ck;
+    for (int32_t v : cand) ck.push_back(Key{distance(p, P.data + (int64_t)v * P.dim, P.dim, P.metric), v});
+    n_dist += (int64_t)cand.size();
+    const bool full = (int)W.size() == L;
+    const Key wmax = W.empty() ? Key{0.f, -1} : *std::prev(W.end());
+    auto selected = [&](const Key& k) { return !(sel && full && wmax < k); };
+    if (lazy) {
+      int64_t n_sel = 0;
+      for (const Key& k : ck) n_sel += selected(k);
+      if (n_sel > 0 && (int64_t)visited.size() + n_sel > P.lazy_cap) {
+        visited.clear();
+        for (const Key& k : W) visited.insert(k.id);
+      }
+    }
+    for (const Key& k : ck) {
+      if (!selected(k)) continue;
+      visited.insert(k.id);
+      W.insert(k);
+    }
+    while ((int)W.size() > L) {
+      const Key w = *std::prev(W.end());
+      W.erase(std::prev(W.end()));
+      popped.erase(w.id);
+      if (del) visited.erase(w.id);
+    }
+  }
+  int i = 0;
+  for (const Key& k : W) {
+    if (i >= P.K) break;
+    if (!popped.count(k.id)) continue;
+    ids_out[i] = k.id;
+    dists_out[i] = k.dist;
+    ++i;
+  }
+  for (; i < P.K; ++i) {
+    ids_out[i] = -1;
+    dists_out[i] = INFINITY;
+  }
+  if (counters) {
+    counters[0] = n_dist;
+    counters[1] = n_exp;
+  }
+  return status;
+}
+
+int search_dispatch(const Problem& P, const float* p, int32_t* ids_out, float* dists_out,
+                    int64_t* counters, trace_fn cb, void* ctx) {
+  if (P.flags & ORACLE_UNION) return search_one_union(P, p, ids_out, dists_out, counters);
+  return search_one(P, p, ids_out, dists_out, counters, cb, ctx);
+}
+
 }  // namespace
 
 extern "C" {
@@ -465,8 +577,8 @@ int64_t oracle_search_steps(const float* data, int64_t n, int32_t dim, const int
   if (nthreads <= 1 || cb) {
     int64_t fails = 0;
     for (int64_t i = 0; i < nq; ++i)
-      fails += search_one(P, queries + i * dim, ids + i * K, dists + i * K,
-                          counters ? counters + 2 * i : nullptr, cb, ctx);
+      fails += search_dispatch(P, queries + i * dim, ids + i * K, dists + i * K,
+                               counters ? counters + 2 * i : nullptr, cb, ctx);
     return fails;
   }
   std::vector<std::thread> pool;
@@ -474,8 +586,8 @@ int64_t oracle_search_steps(const float* data, int64_t n, int32_t dim, const int
   for (int t = 0; t < nthreads; ++t) {
     pool.emplace_back([&, t]() {
       for (int64_t i = t; i < nq; i += nthreads)
-        fails[t] += search_one(P, queries + i * dim, ids + i * K, dists + i * K,
-                               counters ? counters + 2 * i : nullptr, nullptr, nullptr);
+        fails[t] += search_dispatch(P, queries + i * dim, ids + i * K, dists + i * K,
+                                    counters ? counters + 2 * i : nullptr, nullptr, nullptr);
     });
   }
   for (auto& th : pool) th.join();

@@ -62,6 +62,11 @@ int launch_q(song_index* ix, const SearchArgs& a, int qr, int warps, int bps, in
     case 1: return launch_t<NCH, METRIC, VK, 1, MS>(ix, a, warps, bps, sms, st);
     case 2: return launch_t<NCH, METRIC, VK, 2, MS>(ix, a, warps, bps, sms, st);
     case 4: return launch_t<NCH, METRIC, VK, 4, MS>(ix, a, warps, bps, sms, st);
+    case -1:  // reading R17 (one bounded list of q ∪ topk): the hash visited set only
+      if constexpr (VK == VK_HASH && !MS)
+        return launch_t<NCH, METRIC, VK, -1, false>(ix, a, warps, bps, sms, st);
+      else
+        return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH, steps 1");
     default: return launch_t<NCH, METRIC, VK, 0, MS>(ix, a, warps, bps, sms, st);
   }
 }

@@ -113,6 +113,14 @@ __device__ __forceinline__ uint64_t make_key(float d, int id) {
 
 __device__ __forceinline__ int key_id(uint64_t k) { return (int)(uint32_t)(k & 0xffffffffu); }
 
+// Reading R17 keys (the bounded union W): orderable(dist) << 32 | id << 1 |
+// popped — ids < 2^31, so the (dist, id) order is unchanged and the popped
+// mark rides in bit 0 without ever deciding a comparison between two keys
+__device__ __forceinline__ uint64_t make_wkey(float d, int id) {
+  return ((uint64_t)f2ord(d) << 32) | ((uint64_t)(uint32_t)id << 1);
+}
+__device__ __forceinline__ int wkey_id(uint64_t k) { return (int)((uint32_t)(k & 0xffffffffu) >> 1); }
+
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -593,7 +601,7 @@ struct Tier {
   }
   // insert x (warp-uniform, not present) at its sorted position; the caller
   // keeps size < 32 * 64 and within its block budget
-  __device__ __forceinline__ void insert(uint64_t x, int lane) {
+  __device__ __forceinline__ int insert(uint64_t x, int lane) {
     const int n = size, nbk = nb();
     const int pos = rank_warp(x, lane);
     const int b = pos >> 6, o = pos & 63;
@@ -629,6 +637,24 @@ struct Tier {
     }
     __syncwarp();
     size = n + 1;
+    return pos;
+  }
+  // reading R17: set the popped mark (bit 0 of a W key) of element i
+  __device__ __forceinline__ void set_flag(int i, int lane) {
+    const int b = (i >> 6) & 31;
+    const int h = __shfl_sync(FULL, hd, b);
+    if (lane == 0) a[(b << 6) | ((h + i) & 63)] |= 1ull;
+    __syncwarp();
+  }
+  // R17: index of the first element >= i without the popped mark, or size
+  __device__ __forceinline__ int next_unpopped(int i, int lane) const {
+    for (; i < size; i += 32) {
+      const int j = i + lane;
+      const uint64_t v = at(j < size ? j : 0);
+      const unsigned m = __ballot_sync(FULL, j < size && !(v & 1ull));
+      if (m) return i + __ffs(m) - 1;
+    }
+    return size;
   }
   // remove the minimum (element 0)
   __device__ __forceinline__ void pop_front(int lane) {
@@ -1050,6 +1076,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH>::R;
   constexpr bool DEL = (VK == VK_HASH || VK == VK_CUCKOO);  // visited deletion (§IV-E)
+  // QR > 0: q / topk in registers; QR == 0: separate q and topk tiers in
+  // shared memory; QR < 0: reading R17, one bounded list W of q ∪ topk
+  constexpr bool UNQ = QR < 0;
+  constexpr int QRr = QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int L = a.L;
@@ -1064,11 +1094,12 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   uint64_t* keys32 = reinterpret_cast<uint64_t*>(cid + (MS ? 32 * MAX_STEPS : 32));  // 32 keys
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
   // QR == 0 only: q and topk as tiered vectors of ceil(L / 64) blocks
-  const int tslots = QR == 0 ? ((L + 63) >> 6) << 6 : 0;
-  uint64_t* qa = ev + 32;
-  uint64_t* tk = qa + tslots;
+  const int tslots = QR <= 0 ? ((L + 63) >> 6) << 6 : 0;
+  uint64_t* qa = ev + 32;                       // q (or W, R17)
+  uint64_t* tk = qa + tslots;                   // topk (QR == 0 only)
+  const int tkslots = QR == 0 ? tslots : 0;
   int* table = reinterpret_cast<int*>(                                  // 16 B aligned
-      (reinterpret_cast<uintptr_t>(tk + tslots) + 15) & ~uintptr_t(15));
+      (reinterpret_cast<uintptr_t>(tk + tkslots) + 15) & ~uintptr_t(15));
   // 32-bit words of the shared-memory visited table
   const int twords = VK == VK_HASH    ? (1 << a.table_log2)
                      : VK == VK_BLOOM ? ((1 << a.table_log2) >> 5)
@@ -1198,14 +1229,16 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     v_insert_lane0(a.entry);
     int used = 1;  // VK_HASH: live + tombstones; VK_GHASH: live
-    RegArr<QR == 0 ? 1 : QR> q, tk_r;
+    RegArr<QRr> q, tk_r;
     q.clear();
     tk_r.clear();
-    Tier qg{qa, 0, 0}, tg{tk, 0, 0};  // QR == 0
+    Tier qg{qa, 0, 0}, tg{tk, 0, 0};  // QR <= 0 (qg is W when UNQ)
+    int hint = 0;                      // UNQ: index of W's first unpopped key
     if (QR > 0) {
       if (lane == 0) q.v[0] = ke;
     } else {
-      if (lane == 0) qa[0] = ke;
+      if (lane == 0)
+        qa[0] = UNQ ? (ke & ~0xffffffffull) | ((uint64_t)(uint32_t)a.entry << 1) : ke;
       qg.size = 1;
       __syncwarp();
     }
@@ -1221,6 +1254,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     long long st_t = clock64();
 #endif
     while (qsize > 0) {
+      if (UNQ && hint >= qg.size) break;  // R17: no unpopped key left in W
       if (iters >= a.max_iters) {
         capped = true;
         break;
@@ -1231,6 +1265,9 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if (QR > 0) {
         now = __shfl_sync(FULL, q.v[0], 0);
         tmax = tk_r.get(L - 1);  // KEY_MAX unless topk is full
+      } else if (UNQ) {
+        now = qg.at(hint);  // W's smallest unpopped key (R17 step 2)
+        tmax = KEY_MAX;
       } else {
         now = qg.at(0);
         tmax = (tsize == L) ? tg.at(L - 1) : KEY_MAX;
@@ -1244,7 +1281,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if constexpr (VK == VK_CUCKOO) {
         if (QR > 0) {
 #pragma unroll
-          for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) in_topk |= __any_sync(FULL, tk_r.v[r] == now);
+          for (int r = 0; r < QRr; ++r) in_topk |= __any_sync(FULL, tk_r.v[r] == now);
         } else {
           const int r = tg.rank_warp(now, lane);
           const uint64_t at_r = tg.at(r < tsize ? r : 0);
@@ -1254,6 +1291,9 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if (QR > 0) {
         if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
         q.pop_front(lane);
+      } else if (UNQ) {
+        qg.set_flag(hint, lane);  // now moves from "q" to "topk" inside W
+        hint = qg.next_unpopped(hint + 1, lane);
       } else {
         qg.pop_front(lane);
         if (!in_topk) evicted = tg.push1(now, L, lane);
@@ -1264,7 +1304,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       // multi-step probing (§V, R13): up to a.steps pops, each checked
       // against the termination rule with topk as the previous pops left it
       int npop = 1;
-      int popid = key_id(now);  // lane i < npop: id of the i-th popped vertex
+      int popid = UNQ ? wkey_id(now) : key_id(now);  // lane i < npop: id of the i-th popped vertex
       if constexpr (MS) {
         for (; npop < a.steps && npop < qsize; ++npop) {
           const uint64_t nx = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : qg.at(0);
@@ -1343,9 +1383,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       SONG_ST_MARK(2);
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cidg[lane] : -1;
-      uint64_t key = lane < nc ? make_key(dist, myid) : KEY_MAX;
-      const uint64_t thr =
-          (a.sel && tsize == L) ? (QR > 0 ? tk_r.get(L - 1) : tg.at(L - 1)) : KEY_MAX;
+      uint64_t key = lane < nc ? (UNQ ? make_wkey(dist, myid) : make_key(dist, myid)) : KEY_MAX;
+      // selected insertion threshold: topk's max once topk is full;
+      // R17: W's max once W is full
+      const uint64_t thr = UNQ ? ((a.sel && qg.size == L) ? qg.at(L - 1) : KEY_MAX)
+                               : (a.sel && tsize == L)
+                                     ? (QR > 0 ? tk_r.get(L - 1) : tg.at(L - 1))
+                                     : KEY_MAX;
       // selected insertion: filtered only when worse than ALL of topk
       // (a key equal to topk's max can only arise from a filter false negative)
       const bool sel = (lane < nc) && key <= thr;
@@ -1354,10 +1398,12 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if (!sel) key = KEY_MAX;
       // prefetch the adjacency row of the next head = min(q head, best new key)
       if (last_group) {
-        uint64_t qhead = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : (na_g > 0 ? qg.at(0) : KEY_MAX);
+        uint64_t qhead = (QR > 0)  ? __shfl_sync(FULL, q.v[0], 0)
+                         : UNQ     ? (hint < qg.size ? qg.at(hint) : KEY_MAX)
+                         : (na_g > 0 ? qg.at(0) : KEY_MAX);
         uint64_t nxt = umin64(qhead, warp_min_key(key));
         if (nxt != KEY_MAX && lane < a.degree)
-          adjv = __ldg(a.adj + (int64_t)key_id(nxt) * a.degree + lane);
+          adjv = __ldg(a.adj + (int64_t)(UNQ ? wkey_id(nxt) : key_id(nxt)) * a.degree + lane);
         else
           adjv = -1;
       }
@@ -1385,9 +1431,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             __syncwarp();
             if (QR > 0) {
 #pragma unroll
-              for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+              for (int r = 0; r < QRr; ++r) {
                 hs.insert(key_id(q.v[r]), q.v[r] != KEY_MAX);
                 hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
+              }
+            } else if (UNQ) {  // R17: visited := ids(W)
+              for (int i0 = 0; i0 < qg.size; i0 += 32) {
+                const uint64_t kw = qg.at(i0 + lane < qg.size ? i0 + lane : 0);  // (all lanes)
+                hs.insert(wkey_id(kw), i0 + lane < qg.size);
               }
             } else {
               for (int i0 = 0; i0 < na_g; i0 += 32) {
@@ -1399,7 +1450,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
                 hs.insert(key_id(kt), i0 + lane < tsize);
               }
             }
-            used = na_g + tsize;
+            used = UNQ ? qg.size : na_g + tsize;
             __syncwarp();
           }
           const bool took = hs.insert(myid, sel);
@@ -1418,7 +1469,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
               const uint64_t kj = __shfl_sync(FULL, key, j);
               bool dup = false;
 #pragma unroll
-              for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) dup |= __any_sync(FULL, q.v[r] == kj);
+              for (int r = 0; r < QRr; ++r) dup |= __any_sync(FULL, q.v[r] == kj);
               if (dup) qmask &= ~(1u << j);
             }
           }
@@ -1432,10 +1483,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
           const uint64_t sdesc = __shfl_sync(FULL, k2, 31 - lane);  // descending
           // merge into q; evict beyond L (§IV-C) and delete from visited (§IV-E)
           uint64_t out;
-          merge_into<QR == 0 ? 1 : QR>(q, sdesc, lane, out);
+          merge_into<QRr>(q, sdesc, lane, out);
           int ne = 0;  // number of evicted keys (VK_CUCKOO collects them in ev[])
 #pragma unroll
-          for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+          for (int r = 0; r < QRr; ++r) {
             const bool beyond = r * 32 + lane >= L && q.v[r] != KEY_MAX;
             if constexpr (VK == VK_HASH) hs.erase(key_id(q.v[r]), beyond && !a.lazy);
             if constexpr (VK == VK_CUCKOO) {
@@ -1461,6 +1512,36 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             cuckoo_erase_sorted_desc(ne);
           }
         }
+      } else if (UNQ) {  // R17: insert into W, drop its maximum beyond L
+        visit_selected();
+        __syncwarp();
+        if (sel) keys32[__popc(smask & lt)] = key;
+        __syncwarp();
+        key = lane < ns ? keys32[lane] : KEY_MAX;
+        __syncwarp();
+        key = sort_prefix(key, ns, lane);
+        int ne = 0;
+        uint64_t evk = KEY_MAX;  // lane e: the e-th dropped key
+        for (int j = 0; j < ns; ++j) {
+          const uint64_t x = __shfl_sync(FULL, key, j);
+          if (qg.size == L) {
+            const uint64_t mx = qg.at(L - 1);
+            if (x > mx) {  // x and every later key are dropped at once
+              const uint64_t moved = __shfl_sync(FULL, key, (lane - ne + j) & 31);
+              if (lane >= ne && lane < ne + ns - j) evk = moved;
+              ne += ns - j;
+              break;
+            }
+            if (lane == ne) evk = mx;
+            ++ne;
+            qg.size = L - 1;
+            hint = min(hint, qg.size);
+          }
+          const int pos = qg.insert(x, lane);
+          hint = pos <= hint ? pos : hint;  // a new (unpopped) key before the old first one
+        }
+        if constexpr (VK == VK_HASH) hs.erase(wkey_id(evk), lane < ne && !a.lazy);  // [del]
+        qsize_new = qg.size;
       } else {  // QR == 0: the q ring
         visit_selected();
         __syncwarp();
@@ -1538,13 +1619,31 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     // ---- a7: output the first K of topk (Alg. 1 line 17)
     if (QR > 0) {
 #pragma unroll
-      for (int r = 0; r < (QR == 0 ? 1 : QR); ++r) {
+      for (int r = 0; r < QRr; ++r) {
         const int i = r * 32 + lane;
         if (i < a.K) {
           uint64_t k = tk_r.v[r];
           ids_o[i] = (k != KEY_MAX) ? key_id(k) + a.id_offset : -1;
           dists_o[i] = (k != KEY_MAX) ? ord2f((uint32_t)(k >> 32)) : __int_as_float(0x7f800000);
         }
+      }
+    } else if (UNQ) {  // R17: the first K popped keys of W (all of W at a normal stop)
+      int outn = 0;
+      for (int i0 = 0; i0 < qg.size && outn < a.K; i0 += 32) {
+        const int i = i0 + lane;
+        const uint64_t k = qg.at(i < qg.size ? i : 0);
+        const bool pp = i < qg.size && (k & 1ull);
+        const unsigned m = __ballot_sync(FULL, pp);
+        const int o = outn + __popc(m & lt);
+        if (pp && o < a.K) {
+          ids_o[o] = wkey_id(k) + a.id_offset;
+          dists_o[o] = ord2f((uint32_t)(k >> 32));
+        }
+        outn += __popc(m);
+      }
+      for (int i = min(outn, a.K) + lane; i < a.K; i += 32) {
+        ids_o[i] = -1;
+        dists_o[i] = __int_as_float(0x7f800000);
       }
     } else {
       for (int i0 = 0; i0 < a.K; i0 += 32) {

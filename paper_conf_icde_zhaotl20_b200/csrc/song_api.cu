@@ -181,7 +181,8 @@ struct Shape {
   int table_log2;
   int rebuild_at;
   int warp_bytes;
-  int qr;  // register queue width (L <= 32*qr), 0 = shared-memory queues
+  int qr;  // register queue width (L <= 32*qr), 0 = shared-memory tiers, -1 = union (R17)
+  int qk;  // QueueKind
   int nch;
   int warps;  // warps per CTA
 };
@@ -196,11 +197,33 @@ struct Shape {
 #ifndef SONG_HASH_BIG_DEN
 #define SONG_HASH_BIG_DEN 3
 #endif
-int hash_log2_slots(int L) {
+// the bounded union (reading R17) holds <= L + 32 live ids; its table is
+// sized F_u (L + 32), F_u = NUM / DEN
+#ifndef SONG_HASH_UNION_NUM
+#define SONG_HASH_UNION_NUM 8
+#endif
+#ifndef SONG_HASH_UNION_DEN
+#define SONG_HASH_UNION_DEN 3
+#endif
+int hash_log2_slots(int L, bool uni = false) {
+  if (uni)
+    return next_pow2_log2((SONG_HASH_UNION_NUM * (L + 32ll) + SONG_HASH_UNION_DEN - 1) /
+                          SONG_HASH_UNION_DEN);
   const long long live = 2ll * L + 32;
   if (L > 128) return next_pow2_log2((SONG_HASH_BIG_NUM * live + SONG_HASH_BIG_DEN - 1) / SONG_HASH_BIG_DEN);
   const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE : SONG_HASH_FACTOR;
   return next_pow2_log2(F * live);
+}
+
+// the queue structure of a search: registers (L <= 128, separate q / topk),
+// shared-memory tiers (separate q / topk), or the bounded union (R17)
+enum QueueKind { QK_REGS = 0, QK_SEPARATE = 1, QK_UNION = 2 };
+int queue_kind_of(int L, int vk, const song_search_params* p) {
+  const bool union_ok = vk == song::VK_HASH && p->steps <= 1;
+  if (p->queue_kind == SONG_QUEUE_UNION && union_ok) return QK_UNION;
+  if (L <= 128) return QK_REGS;
+  if (p->queue_kind == SONG_QUEUE_AUTO && union_ok) return QK_UNION;
+  return QK_SEPARATE;
 }
 
 Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
@@ -219,6 +242,12 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     // reading R10 default: 4 slots per key of the live bound 2L + 32
     s.table_log2 = p->table_log2 > 0 ? p->table_log2 : next_pow2_log2(4ll * (2 * L + 32)) - 2;
     tbytes = (4 << s.table_log2) * 2;
+  } else if (queue_kind_of(L, vk, p) == QK_UNION) {
+    // R17: live keys <= |W| + 32 new ones <= L + 32; lazy by default
+    s.table_log2 = hash_log2_slots(L, true);
+    s.lazy = p->visited_cap >= 0;
+    s.rebuild_at = s.lazy && p->visited_cap > 0 ? p->visited_cap : (3 << s.table_log2) / 4;
+    tbytes = (1 << s.table_log2) * 4;
   } else {
     // live keys <= |q| + |topk| + 32 new ones <= 2L + 32.  Register-queue
     // sizes get >= 8x (L <= 64) or 4x (L <= 128: a 16 KB table would cut
@@ -240,12 +269,15 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   s.nch = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
   const int rows = s.nch >= 2 ? 4 : SONG_STAGE_ROWS;  // StageRows<NCH>::R
-  s.qr = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 0;
+  const int qk = queue_kind_of(L, vk, p);
+  s.qk = qk;
+  s.qr = qk == QK_UNION ? -1 : qk == QK_SEPARATE ? 0 : L <= 32 ? 1 : L <= 64 ? 2 : 4;
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
   s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
-                 (s.qr == 0 ? 2 * (((L + 63) / 64) * 64) * 8 + 8 : 0) + tbytes;
+                 (s.qr <= 0 ? (s.qr == 0 ? 2 : 1) * (((L + 63) / 64) * 64) * 8 + 8 : 0) +
+                 tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
   // CTA size (1 warp = 1 query): 4 warps unless shared memory is the limit
   s.warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
@@ -286,12 +318,17 @@ int check_params_common(const song_search_params* p, int metric) {
   if (p->max_iters < 0 || p->blocks_per_sm < 0) return fail(SONG_EINVAL, "negative launch parameter");
   if (p->steps < 0) return fail(SONG_EINVAL, "steps %d < 0", p->steps);
   if (p->visited_cap < -1) return fail(SONG_EINVAL, "visited_cap %d < -1", p->visited_cap);
+  if (p->queue_kind < SONG_QUEUE_AUTO || p->queue_kind > SONG_QUEUE_UNION)
+    return fail(SONG_EINVAL, "unknown queue_kind %d", p->queue_kind);
+  if (p->queue_kind == SONG_QUEUE_UNION && (p->visited != SONG_VISITED_HASH || p->steps > 1))
+    return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH and steps <= 1");
   if (p->visited_cap > 0 && p->visited == SONG_VISITED_HASH) {
-    const bool big = p->queue_len > 128;
-    const int slots = 1 << hash_log2_slots(p->queue_len);
-    if (p->visited_cap < 2 * p->queue_len + 32 || p->visited_cap > 3 * (slots / 4))
-      return fail(SONG_EINVAL, "visited_cap %d outside [2L + 32, 3/4 of %d slots]",
-                  p->visited_cap, slots);
+    const bool uni = queue_kind_of(p->queue_len, song::VK_HASH, p) == QK_UNION;
+    const int slots = 1 << hash_log2_slots(p->queue_len, uni);
+    const int lo = uni ? p->queue_len + 32 : 2 * p->queue_len + 32;
+    if (p->visited_cap < lo || p->visited_cap > 3 * (slots / 4))
+      return fail(SONG_EINVAL, "visited_cap %d outside [%d, 3/4 of %d slots]", p->visited_cap,
+                  lo, slots);
   }
   if (p->schedule < SONG_SCHEDULE_AUTO || p->schedule > SONG_SCHEDULE_OUTLIER_FIRST)
     return fail(SONG_EINVAL, "unknown schedule %d", p->schedule);
@@ -759,7 +796,8 @@ int song_search_plan_get(const song_search_params* p, int32_t dim, int32_t metri
   const int vk = vk_of(p);
   out->visited_log2 = sh.table_log2;
   out->visited_cap = vk != song::VK_HASH ? 0 : sh.lazy ? sh.rebuild_at : -1;
-  out->queue_regs = sh.qr;
+  out->queue_regs = sh.qr > 0 ? sh.qr : 0;
+  out->queue_kind = sh.qk;
   out->row_chunks = sh.nch;
   out->smem_per_warp = sh.warp_bytes;
   out->warps_per_block = sh.warps;

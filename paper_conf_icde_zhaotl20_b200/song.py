@@ -44,6 +44,7 @@ class SongError(RuntimeError):
 
 
 SCHEDULES = {"auto": 0, "batch": 1, "outlier_first": 2}  # song.h SONG_SCHEDULE_*
+QUEUE_KINDS = {"auto": 0, "separate": 1, "union": 2}     # song.h SONG_QUEUE_*
 
 
 class SearchParams(ctypes.Structure):
@@ -53,7 +54,7 @@ class SearchParams(ctypes.Structure):
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32),
                 ("steps", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
-                ("schedule", ctypes.c_int32)]
+                ("schedule", ctypes.c_int32), ("queue_kind", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -68,7 +69,7 @@ class SearchPlan(ctypes.Structure):
     _fields_ = [("visited_log2", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
                 ("queue_regs", ctypes.c_int32), ("row_chunks", ctypes.c_int32),
                 ("smem_per_warp", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 2)]
+                ("queue_kind", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 _lib = None
@@ -159,6 +160,7 @@ class Params:
     steps: int = 1  # multi-step probing (pops per iteration, §V)
     visited_cap: int = 0  # hash deletion schedule: 0 lazy (default cap), >0 lazy cap, -1 eager
     schedule: str = "auto"  # ticket order: "auto" | "batch" | "outlier_first"
+    queue_kind: str = "auto"  # "auto" | "separate" (q, topk) | "union" (reading R17)
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -174,6 +176,7 @@ class Params:
         p.steps = self.steps
         p.visited_cap = self.visited_cap
         p.schedule = SCHEDULES[self.schedule]
+        p.queue_kind = QUEUE_KINDS[self.queue_kind]
         return p
 
 

@@ -45,13 +45,23 @@ def song_plan_cap(L, dim, metric):
     return s.default_visited_cap(L, dim, metric)
 
 
-def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0):
-    """The oracle mode matching a GPU search: the hash's deletion schedule is
-    lazy (reading R14) unless visited_cap = -1 or steps > 1 (eager)."""
+def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0, queue_kind="auto"):
+    """The oracle mode matching a GPU search, read from the library's plan
+    (song_search_plan_get): the hash's deletion schedule is lazy (reading
+    R14) unless visited_cap = -1 or steps > 1 (eager), and queues above 128
+    (or queue_kind="union") are the bounded union of reading R17."""
+    from paper_conf_icde_zhaotl20_b200 import song as s
     kw = dict(flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L, log2, visited))
-    if visited == "hash" and steps <= 1 and visited_cap >= 0:
-        kw["flags"] = oracle.OPTIMIZED_LAZY
-        kw["lazy_cap"] = visited_cap or lazy_cap_for(L)
+    if visited == "hash":
+        pl = s.plan(s.Params(K=1, queue_len=L, steps=steps, visited_cap=visited_cap,
+                             queue_kind=queue_kind), 128)
+        flags = oracle.OPTIMIZED
+        if pl.visited_cap > 0:
+            flags |= oracle.LAZY
+            kw["lazy_cap"] = pl.visited_cap
+        if pl.queue_kind == 2:
+            flags |= oracle.UNION
+        kw["flags"] = flags
     if steps > 1:
         kw["steps"] = steps
     return kw
@@ -257,6 +267,32 @@ def test_edges_exact(dim, L, K):
         g = gpu_search(idx, q, K, L, visited)
         o = oracle.search(x, adj, q, K, L, **oracle_kw(visited, L))
         assert_exact(g, o)
+    for qk in ("union", "separate"):  # every queue kind at every L (R17 / §IV-C)
+        for cap in (0, -1):
+            g = gpu_search(idx, q, K, L, "hash", queue_kind=qk, visited_cap=cap)
+            o = oracle.search(x, adj, q, K, L, **oracle_kw("hash", L, visited_cap=cap, queue_kind=qk))
+            assert_exact(g, o)
+
+
+@pytest.mark.parametrize("L", [129, 200, 640, 1280])
+@pytest.mark.parametrize("cap", [0, -1, "min"])
+def test_union_queue_bit_exact(sift100k, L, cap):
+    """Reading R17 (the default above 128): ids, distances and counters
+    bit-exact against the oracle's bounded-union mode, every deletion
+    schedule; results equal the separate q / topk structures (§IV-C)."""
+    cfg, x, q, adj = sift100k
+    cap = L + 32 if cap == "min" else cap
+    s = song()
+    idx = s.SongIndex(x, adj)
+    xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()[:200]
+    g = gpu_search(idx, qn, cfg.K, L, "hash", visited_cap=cap)
+    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap))
+    assert o is not None and s.plan(s.Params(K=1, queue_len=L), 128).queue_kind == 2
+    assert_exact(g, o)
+    sep = gpu_search(idx, qn, cfg.K, L, "hash", queue_kind="separate")
+    np.testing.assert_array_equal(g[0], sep[0])
+    np.testing.assert_array_equal(g[1], sep[1])
+    np.testing.assert_array_equal(g[2][:, 1], sep[2][:, 1])  # the same popped sequence
 
 
 def test_entry_offset_and_unreachable_padding():
@@ -281,8 +317,12 @@ def test_large_queue_len_max():
     o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048))
     assert_exact(g, o)
     g = gpu_search(idx, q[:16], 100, 2048, visited_cap=-1)  # eager deletion
-    o = oracle.search(x, adj, q[:16], 100, 2048)
+    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, visited_cap=-1))
     assert_exact(g, o)
+    for qk in ("separate", "union"):  # both shared-memory queue kinds at the maximum
+        g = gpu_search(idx, q[:16], 100, 2048, queue_kind=qk)
+        o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, queue_kind=qk))
+        assert_exact(g, o)
 
 
 def test_errors():
@@ -371,7 +411,7 @@ def test_deletion_schedules_exact(sift100k, L, cap):
     g = gpu_search(idx, qn, cfg.K, L, "hash", visited_cap=cap)
     o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap))
     assert_exact(g, o)
-    eager = oracle.search(xn, an, qn, cfg.K, L, nthreads=8)
+    eager = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=-1))
     np.testing.assert_array_equal(g[0], eager[0])  # the schedule never changes results
     np.testing.assert_array_equal(g[1], eager[1])
     if cap != -1:
