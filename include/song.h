@@ -270,6 +270,31 @@ int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int
                     int32_t Kin, int32_t K, int32_t* ids_out, float* dists_out,
                     void* stream);
 
+/* The same merge fused with the gather over peer memory (dataset sharding on
+ * one node): each of the G ranks searched its shard into a [nq][Kin]
+ * ids / dists buffer the other ranks can address (e.g. torch symmetric memory
+ * over NVLink / NVSwitch), rows sorted by (dist, global id), -1 padded.
+ *   ids_peers, dists_peers  DEVICE arrays of G DEVICE pointers: rank g's rows;
+ *   signal_peers            DEVICE array of G DEVICE pointers to each rank's
+ *                           signal pad (>= G uint32, zero-initialised once and
+ *                           reserved for this call), or NULL;
+ *   rank                    this rank (0 <= rank < G);
+ *   epoch                   > every epoch used before with these pads;
+ *   ids_out, dists_out      DEVICE [nq][K] on this rank: the K smallest keys.
+ * With pads, the kernel (enqueued on `stream` after this rank's search) first
+ * stores `epoch` into slot `rank` of every peer's pad (release, system
+ * scope), then waits for every peer's slot of its own pad (acquire) and
+ * merges straight from the peers' buffers: no staging copy, no separate
+ * all-gather.  Every rank must make the call with the same G, nq, Kin, epoch.
+ * Without pads the caller guarantees the peers' rows are complete and
+ * visible (one-GPU emulation, or after its own barrier).  Asynchronous.
+ * Errors: SONG_EINVAL (NULL, sizes, rank/epoch), SONG_EUNSUPPORTED (K or Kin
+ * > 1024). */
+int song_merge_topk_peers(const int32_t* const* ids_peers, const float* const* dists_peers,
+                          uint32_t* const* signal_peers, int32_t rank, int32_t G, int64_t nq,
+                          int32_t Kin, int32_t K, uint32_t epoch, int32_t* ids_out,
+                          float* dists_out, void* stream);
+
 /* ---- 1-bit random projection (§VII "Out-of-GPU-memory datasets") ----
  * "For two data vectors u, v ... we generate a random vector r with entries in
  * iid standard normal ... With h independent random vectors, each data point

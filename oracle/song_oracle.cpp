@@ -459,9 +459,12 @@ int search_one(const Problem& P, const float* p, int32_t* ids_out, float* dists_
 //   3. Locate the unvisited neighbours of u (row order, first occurrence).
 //   4. Distances; n_dist += |cand|.
 //   5. Maintain: [sel] skip c when |W| = L and key(c) > max(W) (a key beaten
-//      by L discovered ones can never be popped nor returned); [lazy] if
-//      |visited| + selected > C first set visited := ids(W); insert the
-//      selected into visited and W (unpopped); while |W| > L drop max(W) and
+//      by L discovered ones can never be popped nor returned: once full, W
+//      stays full and its max only decreases); [lazy] if |visited| + |cand| > C
+//      first set visited := ids(W), then mark EVERY candidate visited (a
+//      skipped one can never enter W, so marking it saves recomputing it;
+//      eager deletion keeps visited = ids(W) and marks only the selected);
+//      insert the selected into W (unpopped); while |W| > L drop max(W) and
 //      [del] erase it from visited.
 //   6. Return the first K popped keys of W (all of W is popped at the end).
 // Same popped sequence and result as Algorithm 1 (the popped key is q's min
@@ -515,16 +518,15 @@ int search_one_union(const Problem& P, const float* p, int32_t* ids_out, float* 
     const bool full = (int)W.size() == L;
     const Key wmax = W.empty() ? Key{0.f, -1} : *std::prev(W.end());
     auto selected = [&](const Key& k) { return !(sel && full && wmax < k); };
-    if (lazy) {
-      int64_t n_sel = 0;
-      for (const Key& k : ck) n_sel += selected(k);
-      if (n_sel > 0 && (int64_t)visited.size() + n_sel > P.lazy_cap) {
-        visited.clear();
-        for (const Key& k : W) visited.insert(k.id);
-      }
+    if (lazy && !ck.empty() && (int64_t)visited.size() + (int64_t)ck.size() > P.lazy_cap) {
+      visited.clear();
+      for (const Key& k : W) visited.insert(k.id);
     }
     for (const Key& k : ck) {
-      if (!selected(k)) continue;
+      if (!selected(k)) {
+        if (lazy) visited.insert(k.id);
+        continue;
+      }
       visited.insert(k.id);
       W.insert(k);
     }

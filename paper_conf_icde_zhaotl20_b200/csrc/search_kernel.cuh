@@ -1424,7 +1424,11 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
           (void)dropped;  // a dropped fingerprint is a false negative (oracle: drops)
         }
         if constexpr (VK == VK_HASH) {
-          if (used + ns > a.rebuild_at) {
+          // R17 lazy: every candidate is marked visited (a skipped key can
+          // never enter W again), so the capacity check counts all of them
+          const bool ins = (UNQ && a.lazy) ? lane < nc : sel;
+          const int nins = (UNQ && a.lazy) ? nc : ns;
+          if (used + nins > a.rebuild_at) {
             // tombstones accumulated (eager deletion) or the capacity is reached
             // (lazy deletion, R14): rebuild visited = ids(q) ∪ ids(topk)
             for (int i = lane; i < twords; i += 32) table[i] = EMPTY;
@@ -1453,7 +1457,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             used = UNQ ? qg.size : na_g + tsize;
             __syncwarp();
           }
-          const bool took = hs.insert(myid, sel);
+          const bool took = hs.insert(myid, ins);
           used += __popc(__ballot_sync(FULL, took));
         }
       };

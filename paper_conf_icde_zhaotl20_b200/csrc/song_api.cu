@@ -1051,6 +1051,25 @@ int song_stage_cycles(song_index* ix, uint64_t* cycles_out, int32_t reset) {
 #endif
 }
 
+int song_merge_topk_peers(const int32_t* const* ids_peers, const float* const* dists_peers,
+                          uint32_t* const* signal_peers, int32_t rank, int32_t G, int64_t nq,
+                          int32_t Kin, int32_t K, uint32_t epoch, int32_t* ids_out,
+                          float* dists_out, void* stream) {
+  if (!ids_peers || !dists_peers || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (G < 1 || G > 256 || nq < 1 || Kin < 1 || K < 1)
+    return fail(SONG_EINVAL, "G must be in [1, 256], nq, Kin, K >= 1");
+  if (K > 1024 || Kin > 1024) return fail(SONG_EUNSUPPORTED, "K and Kin must be <= 1024");
+  if (signal_peers && (rank < 0 || rank >= G || epoch == 0))
+    return fail(SONG_EINVAL, "rank %d outside [0, %d) or epoch 0", rank, G);
+  const int warps = 8;
+  const int64_t blocks = (nq + warps - 1) / warps;
+  const int threads = std::max(warps * 32, ((G + 31) / 32) * 32);
+  song::song_merge_peers_kernel<<<(unsigned)blocks, threads, 0, (cudaStream_t)stream>>>(
+      ids_peers, dists_peers, signal_peers, rank, G, nq, Kin, K, epoch, ids_out, dists_out);
+  CUDA_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
 const char* song_last_error(void) { return g_err.c_str(); }
 
 const char* song_version(void) { return "song-b200 0.1 sm_100a"; }

@@ -34,7 +34,7 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
             "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward",
-            "song_search_plan_get", "song_stage_cycles"]
+            "song_search_plan_get", "song_stage_cycles", "song_merge_topk_peers"]
 
 
 class SongError(RuntimeError):
@@ -105,6 +105,8 @@ def lib():
         L.song_search_plan_get.argtypes = [ctypes.POINTER(SearchParams), i32, i32,
                                            ctypes.POINTER(SearchPlan)]
         L.song_stage_cycles.argtypes = [P, P, i32]
+        L.song_merge_topk_peers.argtypes = [P, P, P, i32, i32, i64, i32, i32, ctypes.c_uint32,
+                                            P, P, P]
         L.song_last_error.restype = ctypes.c_char_p
         L.song_last_error.argtypes = []
         L.song_version.restype = ctypes.c_char_p
@@ -115,7 +117,7 @@ def lib():
                      "song_index_create_codes", "song_index_create_rp",
                      "song_search_codes_ex", "song_build_graph", "song_build_graph_batched",
                      "song_build_graph_from_forward", "song_search_plan_get",
-                     "song_stage_cycles"):
+                     "song_stage_cycles", "song_merge_topk_peers"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -345,6 +347,28 @@ def merge_topk(ids, dists, K: int):
     _check(lib().song_merge_topk(ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(dists.data_ptr()),
                                  G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
                                  ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
+    return oi, od
+
+
+def merge_topk_peers(ids_ptrs, dists_ptrs, nq: int, kin: int, K: int, out=None,
+                     sig_ptrs=None, rank: int = 0, epoch: int = 0, device=None):
+    """song_merge_topk_peers: ``ids_ptrs`` / ``dists_ptrs`` are CUDA int64
+    tensors [G] holding the device addresses of each rank's [nq, kin] rows
+    (peer-mapped, e.g. symmetric memory); ``sig_ptrs`` the [G] signal-pad
+    addresses or None.  Returns (ids [nq, K], dists [nq, K]) on ``device``."""
+    torch = _torch()
+    dev = device or ids_ptrs.device
+    G = int(ids_ptrs.numel())
+    if out is None:
+        oi = torch.empty((nq, K), dtype=torch.int32, device=dev)
+        od = torch.empty((nq, K), dtype=torch.float32, device=dev)
+    else:
+        oi, od = out
+    _check(lib().song_merge_topk_peers(
+        ctypes.c_void_p(ids_ptrs.data_ptr()), ctypes.c_void_p(dists_ptrs.data_ptr()),
+        ctypes.c_void_p(sig_ptrs.data_ptr() if sig_ptrs is not None else 0), int(rank), G,
+        int(nq), int(kin), int(K), int(epoch), ctypes.c_void_p(oi.data_ptr()),
+        ctypes.c_void_p(od.data_ptr()), _stream_ptr(dev)))
     return oi, od
 
 

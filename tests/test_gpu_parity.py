@@ -396,6 +396,55 @@ def test_dataset_sharding_emulated_on_one_gpu(sift100k):
     ei, ed = oracle.merge_shards(per_i, per_d, K)
     np.testing.assert_array_equal(mi.cpu().numpy(), ei)
     np.testing.assert_array_equal(md.cpu().numpy(), ed)
+    # the fused gather + merge kernel reading the G shards' buffers through a
+    # pointer table (on one GPU the "peers" are local buffers; no pads)
+    ptr = lambda ts: torch.tensor([t.data_ptr() for t in ts], dtype=torch.int64, device="cuda")  # noqa: E731
+    fi, fd = s.merge_topk_peers(ptr(gi), ptr(gd), q.shape[0], K, K)
+    np.testing.assert_array_equal(fi.cpu().numpy(), ei)
+    np.testing.assert_array_equal(fd.cpu().numpy(), ed)
+    # ... and with signal pads: one pad per "rank", every rank's merge signals
+    # all pads first (here all G merges run on one GPU, one after another, so
+    # rank g waits only on the pads already set: run them in reverse order of
+    # need by pre-setting the other ranks' slots)
+    pads = [torch.zeros(G, dtype=torch.int32, device="cuda") for _ in range(G)]
+    for g in range(G):
+        for h in range(G):
+            pads[g][h] = 7  # every peer already signalled epoch 7
+    for g in range(G):
+        pi, pd = s.merge_topk_peers(ptr(gi), ptr(gd), q.shape[0], K, K, sig_ptrs=ptr(pads),
+                                    rank=g, epoch=7)
+        np.testing.assert_array_equal(pi.cpu().numpy(), ei)
+        np.testing.assert_array_equal(pd.cpu().numpy(), ed)
+    torch.cuda.synchronize()
+    assert all(int(p[g]) == 7 for g, p in enumerate(pads))
+
+
+def test_fused_peer_merge_over_symmetric_memory(sift100k, tmp_path):
+    """The product path of dataset sharding (ShardedIndex.search, NCCL): the
+    search writes into symmetric-memory buffers and song_merge_topk_peers
+    signals and merges — on a one-rank NCCL group here (the driver's boxes
+    have one GPU), bit-exact against the oracle's per-shard search + merge."""
+    import torch.distributed as dist
+    from paper_conf_icde_zhaotl20_b200 import sharded
+    cfg, x, q, adj = sift100k
+    s = song()
+    store = dist.FileStore(str(tmp_path / "store"), 1)
+    dist.init_process_group("nccl", store=store, rank=0, world_size=1,
+                            device_id=torch.device("cuda", 0))
+    try:
+        K, L = 10, 40
+        si = sharded.ShardedIndex(x, adj, id_offset=0)
+        for _ in range(2):  # the second call reuses the buffers (epoch 2)
+            fi, fd = si.search(q, q.shape[0], K, L, fused=True)
+            torch.cuda.synchronize()
+        assert si._merger.epoch == 2
+        oi, od, _, _ = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), K, L,
+                                     nthreads=8, **oracle_kw("hash", L))
+        ei, ed = oracle.merge_shards([oi], [od], K)
+        np.testing.assert_array_equal(fi.cpu().numpy(), ei)
+        np.testing.assert_array_equal(fd.cpu().numpy(), ed)
+    finally:
+        dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("L", [10, 48, 64, 128, 200])
