@@ -328,8 +328,9 @@ def ground_truth(x, q, K, metric):
     torch.backends.cuda.matmul.allow_tf32 = False
     out = []
     xn2 = (x * x).sum(1)
-    for s in range(0, q.shape[0], 1024):
-        qq = q[s:s + 1024]
+    step = int(max(1, min(1024, (1 << 30) // max(1, x.shape[0]))))  # <= 4 GiB of distances
+    for s in range(0, q.shape[0], step):
+        qq = q[s:s + step]
         if metric == "l2":
             d = (qq * qq).sum(1, keepdim=True) + xn2[None] - 2 * qq @ x.T
         elif metric == "ip":
@@ -337,7 +338,10 @@ def ground_truth(x, q, K, metric):
         else:
             d = 1 - (qq / qq.norm(dim=1, keepdim=True)) @ (x / x.norm(dim=1, keepdim=True)).T
         out.append(torch.topk(d, K, dim=1, largest=False).indices)
-    return torch.cat(out).int()
+        del d
+    res = torch.cat(out).int()
+    torch.cuda.empty_cache()  # the libsong allocations that follow use cudaMalloc directly
+    return res
 
 
 def recall_t(ids, truth):

@@ -54,6 +54,10 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--max-L", type=int, default=512)
+    ap.add_argument("--config", default="mnist1m", choices=["mnist1m", "mnist8m"])
+    ap.add_argument("--builder", default="exact", choices=["exact", "batched"],
+                    help="graph on the original vectors: exact insertion (workloads.graph, "
+                         "O(n^2)) or the library's batched-insertion builder (R16; MNIST8m)")
     ap.add_argument("--out", default="")
     args = ap.parse_args()
 
@@ -64,16 +68,22 @@ def main():
     from workloads.synth import CONFIGS, MnistLike, rp_matrix
 
     log = lambda m: print(f"[bench_rp] {m}", file=sys.stderr, flush=True)  # noqa: E731
-    cfg = CONFIGS["mnist1m"]
+    cfg = CONFIGS[args.config]
     dev = torch.device("cuda", 0)
     t0 = time.time()
     gen = MnistLike(cfg.dim, cfg.seed, dev)
     x = gen.sample(args.n, cfg.seed)
     q = gen.sample(args.nq, cfg.seed + 1)
-    adj = build_graph(x, degree=cfg.degree, metric="l2")
+    if args.builder == "batched":
+        b = bench.BUILD
+        adj = song.build_graph_batched(x, cfg.degree, "l2", prefix=b["prefix"],
+                                       queue_len=b["queue_len"], batch_shift=b["batch_shift"])
+    else:
+        adj = build_graph(x, degree=cfg.degree, metric="l2")
     torch.cuda.synchronize()
     log(f"data + graph {time.time() - t0:.1f}s")
     truth = bench.ground_truth(x, q, 1, "l2")
+    torch.cuda.empty_cache()
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     def curve(idx, label, bytes_per_dist, ham_truth=None):
@@ -113,9 +123,10 @@ def main():
                 break
         return pts
 
-    result = {"figure": "Fig. 14 (P:1823) on B200", "workload":
-              f"MNIST1m-shaped: {args.n}x784 integer pixels, L2, degree-32 graph on the "
-              f"original vectors, {args.nq} queries, top-1", "curves": {}, "encode": {}}
+    result = {"figure": "Fig. 14 (P:1823) / Table IV (P:1827-1831) on B200", "workload":
+              f"{cfg.name}-shaped: {args.n}x784 integer pixels, L2, degree-32 graph "
+              f"({args.builder} builder) on the original vectors, {args.nq} queries, top-1",
+              "curves": {}, "encode": {}}
     # original vectors ("SONG" line of Fig. 14)
     idx = song.SongIndex(x, adj, metric="l2")
     result["curves"]["original-784"] = curve(idx, "original", 4 * 784)
