@@ -195,7 +195,10 @@ typedef struct song_search_plan {
   int32_t warps_per_block; /* CTA size of the persistent grid (1 warp = 1 query) */
   int32_t queue_kind;      /* 0 registers, 1 separate shared-memory q and topk, 2 the
                               bounded union of reading R17 (song_search_params.queue_kind) */
-  int32_t reserved;        /* 0 */
+  int32_t visited_global;  /* 1: the hash visited table of each warp lives in global
+                              memory (L2) instead of shared memory — chosen for the
+                              bounded union when it lets >= 1.5x the warps reside on an
+                              SM; 0 otherwise */
 } song_search_plan;
 
 /* Errors: SONG_EINVAL (NULL, bad params as song_search_ex would report them,

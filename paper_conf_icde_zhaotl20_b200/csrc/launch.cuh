@@ -49,6 +49,18 @@ int launch_t(song_index* ix, SearchArgs a, int warps, int blocks_per_sm, int num
     int rc = prepare_global_tables(ix, a, grid * warps, st);
     if (rc) return rc;
   }
+  if (QR == -2) {  // per-warp visited tables in global memory (cleared by the kernel)
+    const size_t need = (size_t)grid * warps * ((size_t)4 << a.table_log2);
+    if (need > ix->gvis_bytes) {
+      CUDA_TRY(cudaStreamSynchronize(st));
+      cudaFree(ix->d_gvis);
+      ix->d_gvis = nullptr;
+      ix->gvis_bytes = 0;
+      CUDA_TRY(cudaMalloc(&ix->d_gvis, need));
+      ix->gvis_bytes = need;
+    }
+    a.gvis = ix->d_gvis;
+  }
   CUDA_TRY(cudaMemsetAsync(a.ticket, 0, sizeof(unsigned), st));
   kern<<<(unsigned)grid, warps * 32, smem, st>>>(a);
   CUDA_TRY(cudaGetLastError());
@@ -63,10 +75,13 @@ int launch_q(song_index* ix, const SearchArgs& a, int qr, int warps, int bps, in
     case 2: return launch_t<NCH, METRIC, VK, 2, MS>(ix, a, warps, bps, sms, st);
     case 4: return launch_t<NCH, METRIC, VK, 4, MS>(ix, a, warps, bps, sms, st);
     case -1:  // reading R17 (one bounded list of q ∪ topk): the hash visited set only
-      if constexpr (VK == VK_HASH && !MS)
+    case -2:  // ... with the visited table in global memory
+      if constexpr (VK == VK_HASH && !MS) {
+        if (qr == -2) return launch_t<NCH, METRIC, VK, -2, false>(ix, a, warps, bps, sms, st);
         return launch_t<NCH, METRIC, VK, -1, false>(ix, a, warps, bps, sms, st);
-      else
+      } else {
         return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH, steps 1");
+      }
     default: return launch_t<NCH, METRIC, VK, 0, MS>(ix, a, warps, bps, sms, st);
   }
 }

@@ -74,6 +74,7 @@ struct SearchArgs {
   uint32_t gen0;   // VK_GHASH: generation base of this launch
   int warp_smem_bytes;
   unsigned long long* stage_cycles;  // SONG_STAGE_TIMING builds: [4] SM cycles per stage
+  int* gvis;       // QR == -2: [grid warps][2^table_log2] int32 visited tables (global)
 };
 
 // SONG_STAGE_TIMING (a separate build, never the product library): lane 0 of
@@ -152,14 +153,26 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
 // so up to 32 operations proceed in parallel, and all loops are
 // warp-collective (trip count decided by __any_sync) so the warp stays
 // converged for the shuffles that follow.
-struct HashSet {
+// GLOBAL: the table lives in a per-warp region of global memory (L2-resident;
+// the bounded union at large queue_len, where a shared-memory table would
+// cost most of the SM's resident warps): buckets are read at L2 (ld.cg), so
+// the reads see the atomicCAS / store results of the same warp.
+template <bool GLOBAL = false>
+struct HashSetT {
   int* slot;
   int log2;  // slots = 2^log2, buckets = 2^(log2 - 2)
   __device__ __forceinline__ unsigned home(int v) const {
     return ((uint32_t)v * 0x9E3779B1u) >> (34 - log2);
   }
   __device__ __forceinline__ int4 bucket(unsigned b) const {
+    if constexpr (GLOBAL) return __ldcg(reinterpret_cast<const int4*>(slot) + b);
     return reinterpret_cast<const int4*>(slot)[b];
+  }
+  // every slot EMPTY (warp-collective; 16 B stores)
+  __device__ __forceinline__ void clear(int lane) {
+    int4* s4 = reinterpret_cast<int4*>(slot);
+    for (int i = lane; i < (1 << (log2 - 2)); i += 32) s4[i] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
+    __syncwarp();
   }
   // membership of v for lanes with act; result false elsewhere
   __device__ __forceinline__ bool contains(int v, bool act) const {
@@ -171,6 +184,26 @@ struct HashSet {
         const int4 s = bucket(b);
         found = (s.x == v) | (s.y == v) | (s.z == v) | (s.w == v);
         const bool open = (s.x == EMPTY) | (s.y == EMPTY) | (s.z == EMPTY) | (s.w == EMPTY);
+        act = !found && !open;
+        b = (b + 1) & mask;
+      }
+    }
+    return found;
+  }
+  // contains(), also returning (eslot) the first EMPTY slot of the bucket the
+  // probe ended in — where an insert of v would go — or -1 when v was found
+  __device__ __forceinline__ bool contains_slot(int v, bool act, int& eslot) const {
+    const unsigned mask = (1u << (log2 - 2)) - 1;
+    unsigned b = home(v);
+    bool found = false;
+    eslot = -1;
+    while (__any_sync(FULL, act)) {
+      if (act) {
+        const int4 s = bucket(b);
+        found = (s.x == v) | (s.y == v) | (s.z == v) | (s.w == v);
+        const bool e0 = s.x == EMPTY, e1 = s.y == EMPTY, e2 = s.z == EMPTY, e3 = s.w == EMPTY;
+        const bool open = e0 | e1 | e2 | e3;
+        if (!found && open) eslot = 4 * (int)b + (e0 ? 0 : e1 ? 1 : e2 ? 2 : 3);
         act = !found && !open;
         b = (b + 1) & mask;
       }
@@ -220,6 +253,8 @@ struct HashSet {
     }
   }
 };
+
+using HashSet = HashSetT<false>;
 
 // Bloom filter with the k = 7 double-hashing spec of reading A8:
 // bit_i = (h1 + i*h2) mod m, h1 = fmix32(id), h2 = fmix32(id ^ 0x5bd1e995) | 1.
@@ -1079,6 +1114,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   // QR > 0: q / topk in registers; QR == 0: separate q and topk tiers in
   // shared memory; QR < 0: reading R17, one bounded list W of q ∪ topk
   constexpr bool UNQ = QR < 0;
+  constexpr bool GVT = QR == -2;  // R17 with the visited table in global memory
   constexpr int QRr = QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
@@ -1095,17 +1131,19 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
   // QR == 0 only: q and topk as tiered vectors of ceil(L / 64) blocks
   const int tslots = QR <= 0 ? ((L + 63) >> 6) << 6 : 0;
-  uint64_t* qa = ev + 32;                       // q (or W, R17)
+  int* cslot = reinterpret_cast<int*>(ev + 32);  // GVT: each candidate's insert slot
+  uint64_t* qa = reinterpret_cast<uint64_t*>(cslot + 32);  // q (or W, R17)
   uint64_t* tk = qa + tslots;                   // topk (QR == 0 only)
   const int tkslots = QR == 0 ? tslots : 0;
-  int* table = reinterpret_cast<int*>(                                  // 16 B aligned
-      (reinterpret_cast<uintptr_t>(tk + tkslots) + 15) & ~uintptr_t(15));
+  int* table = GVT ? a.gvis + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2)
+                  : reinterpret_cast<int*>(                             // 16 B aligned
+                        (reinterpret_cast<uintptr_t>(tk + tkslots) + 15) & ~uintptr_t(15));
   // 32-bit words of the shared-memory visited table
   const int twords = VK == VK_HASH    ? (1 << a.table_log2)
                      : VK == VK_BLOOM ? ((1 << a.table_log2) >> 5)
                      : VK == VK_CUCKOO ? (2 << a.table_log2)  // 4 x u16 per bucket
                                        : 0;
-  HashSet hs{table, a.table_log2};
+  HashSetT<GVT> hs{table, a.table_log2};
   BloomSet bs{reinterpret_cast<uint32_t*>(table), a.table_log2};
   CuckooSet cs{reinterpret_cast<uint16_t*>(table), a.table_log2};
   GHash gh{a.gtab + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2),
@@ -1221,7 +1259,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     }
 
     // ---- a2: init — visited = {e}, q = {(d_e, e)}, topk = {} (Alg. 1 line 1)
-    for (int i = lane; i < twords; i += 32) table[i] = VK == VK_HASH ? EMPTY : 0;
+    if constexpr (VK == VK_HASH)
+      hs.clear(lane);
+    else
+      for (int i = lane; i < twords; i += 32) table[i] = 0;
     if (VK == VK_GHASH) gh.gen = ++gen;  // a fresh generation empties the table
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
@@ -1335,11 +1376,17 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
         keep = keep && ((grp & lt) == 0);
       }
       // (called by every lane: the probe loops are warp-collective)
-      const bool seen = v_contains(v, keep);
+      int eslot = -1;
+      bool seen;
+      if constexpr (GVT)  // remember where each candidate's insert goes (one L2 trip less)
+        seen = hs.contains_slot(v, keep, eslot);
+      else
+        seen = v_contains(v, keep);
       keep = keep && !seen;
       const unsigned km = __ballot_sync(FULL, keep);
       int nc_all = __popc(km);
       if (keep) cid[__popc(km & lt)] = v;
+      if (GVT && keep) cslot[__popc(km & lt)] = eslot;
       __syncwarp();
       if constexpr (MS) {
         // the other popped rows, in pop order: one candidate list (R13)
@@ -1428,10 +1475,12 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
           // never enter W again), so the capacity check counts all of them
           const bool ins = (UNQ && a.lazy) ? lane < nc : sel;
           const int nins = (UNQ && a.lazy) ? nc : ns;
+          bool rebuilt = false;
           if (used + nins > a.rebuild_at) {
+            rebuilt = true;
             // tombstones accumulated (eager deletion) or the capacity is reached
             // (lazy deletion, R14): rebuild visited = ids(q) ∪ ids(topk)
-            for (int i = lane; i < twords; i += 32) table[i] = EMPTY;
+            hs.clear(lane);
             __syncwarp();
             if (QR > 0) {
 #pragma unroll
@@ -1457,8 +1506,21 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             used = UNQ ? qg.size : na_g + tsize;
             __syncwarp();
           }
-          const bool took = hs.insert(myid, ins);
-          used += __popc(__ballot_sync(FULL, took));
+          if (GVT && a.lazy && !rebuilt) {
+            // the locate probe left each candidate's slot (the first EMPTY of
+            // the bucket its probe ended in): one plain store per candidate,
+            // the lowest lane of a shared slot wins, the others probe again
+            const int es = ins ? cslot[lane] : -1 - lane;
+            const unsigned grp = __match_any_sync(FULL, es);
+            const bool win = ins && es >= 0 && (grp & lt) == 0;
+            if (win) table[es] = myid;
+            __syncwarp();
+            const bool took = hs.insert(myid, ins && !win);
+            used += __popc(__ballot_sync(FULL, took || win));
+          } else {
+            const bool took = hs.insert(myid, ins);
+            used += __popc(__ballot_sync(FULL, took));
+          }
         }
       };
       int qsize_new = min(na_g + ns, L);

@@ -137,6 +137,7 @@ void free_index(song_index* ix) {
   cudaFree(ix->d_ids);
   cudaFree(ix->d_dists);
   cudaFree(ix->d_gtab);
+  cudaFree(ix->d_gvis);
   cudaFree(ix->d_R);
   cudaFree(ix->d_centroid);
   cudaFreeHost(ix->h_status);
@@ -183,6 +184,7 @@ struct Shape {
   int warp_bytes;
   int qr;  // register queue width (L <= 32*qr), 0 = shared-memory tiers, -1 = union (R17)
   int qk;  // QueueKind
+  int gvis;  // 1: the visited table in global memory (R17, QR == -2)
   int nch;
   int warps;  // warps per CTA
 };
@@ -275,14 +277,27 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
-  s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 +
+  s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 + 32 * 4 +
                  (s.qr <= 0 ? (s.qr == 0 ? 2 : 1) * (((L + 63) / 64) * 64) * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
+  s.gvis = 0;
+  if (s.qr == -1) {
+    // R17 at large queue_len: the visited table moves to global memory (L2)
+    // when that holds >= 1.5x the resident warps per SM (the union kernels
+    // use <= 80 registers: at most 24 warps per SM)
+    auto resident = [](int wb) { return std::min(24, (int)((227 * 1024) / (wb + 256))); };
+    const int wb0 = ((s.warp_bytes - tbytes) + 127) & ~127;
+    if (2 * resident(wb0) >= 3 * resident(s.warp_bytes)) {
+      s.gvis = 1;
+      s.qr = -2;
+      s.warp_bytes = wb0;
+    }
+  }
   // CTA size (1 warp = 1 query): 4 warps unless shared memory is the limit
   s.warps = p->warps_per_block > 0 ? p->warps_per_block : 4;
   while (s.warps > 1 && (size_t)s.warp_bytes * s.warps > 200 * 1024) s.warps >>= 1;
-  if (p->warps_per_block <= 0 && s.warp_bytes > 16 * 1024) {
+  if (p->warps_per_block <= 0) {
     // shared-memory-bound queue lengths: the CTA size that keeps the most warps
     // resident (227 KB per SM; e.g. 73 KB per warp at L = 1536: 1-warp CTAs
     // hold 3 warps per SM where 2-warp CTAs hold 2)
@@ -443,6 +458,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   a.gtab = nullptr;
   a.gen0 = 0;
   a.stage_cycles = nullptr;
+  a.gvis = nullptr;
 #ifdef SONG_STAGE_TIMING
   if (!ix->d_stage) {
     CUDA_TRY(cudaMalloc(&ix->d_stage, 4 * sizeof(unsigned long long)));
@@ -652,6 +668,7 @@ void free_search_view(song_index* view) {
   cudaFree(view->d_ticket);
   cudaFree(view->d_status);
   cudaFree(view->d_gtab);
+  cudaFree(view->d_gvis);
   cudaFree(view->d_order);
   cudaFree(view->d_qbin);
   cudaFree(view->d_bins);
@@ -798,6 +815,7 @@ int song_search_plan_get(const song_search_params* p, int32_t dim, int32_t metri
   out->visited_cap = vk != song::VK_HASH ? 0 : sh.lazy ? sh.rebuild_at : -1;
   out->queue_regs = sh.qr > 0 ? sh.qr : 0;
   out->queue_kind = sh.qk;
+  out->visited_global = sh.gvis;
   out->row_chunks = sh.nch;
   out->smem_per_warp = sh.warp_bytes;
   out->warps_per_block = sh.warps;

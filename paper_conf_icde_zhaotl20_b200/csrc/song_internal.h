@@ -23,6 +23,8 @@ struct song_index {
   uint64_t* d_gtab = nullptr;          // global visited tables (HASH_GLOBAL kinds)
   size_t gtab_bytes = 0;
   uint64_t gen_next = 1;               // next generation base for d_gtab
+  int* d_gvis = nullptr;               // R17 global visited tables (QR == -2)
+  size_t gvis_bytes = 0;
   cudaStream_t stream = nullptr;       // owned; used by song_search
   cudaStream_t last_stream = nullptr;  // stream of the last search
   cudaEvent_t last_done = nullptr;     // recorded after the last search's kernels

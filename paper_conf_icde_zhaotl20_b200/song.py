@@ -69,7 +69,7 @@ class SearchPlan(ctypes.Structure):
     _fields_ = [("visited_log2", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
                 ("queue_regs", ctypes.c_int32), ("row_chunks", ctypes.c_int32),
                 ("smem_per_warp", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
-                ("queue_kind", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("queue_kind", ctypes.c_int32), ("visited_global", ctypes.c_int32)]
 
 
 _lib = None
