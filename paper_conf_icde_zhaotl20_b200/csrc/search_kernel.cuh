@@ -638,41 +638,54 @@ struct Tier {
   // keeps size < 32 * 64 and within its block budget
   __device__ __forceinline__ int insert(uint64_t x, int lane) {
     const int n = size, nbk = nb();
-    const int pos = rank_warp(x, lane);
-    const int b = pos >> 6, o = pos & 63;
-    // reads: the last key of every full block >= b (it moves to the next block)
-    const bool full = ((lane + 1) << 6) <= n;
-    const uint64_t v = (lane >= b && lane < nbk && full) ? a[(lane << 6) | ((hd + 63) & 63)] : 0;
-    const uint64_t vin = __shfl_up_sync(FULL, v, 1);  // lane c: the key block c - 1 passes on
-    const int hb = __shfl_sync(FULL, hd, b & 31);
-    const int cnt = b < nbk ? min(64, n - (b << 6)) : 0;
+    if (nbk == 0) {  // empty: x opens block 0
+      if (lane == 0) {
+        hd = 0;
+        a[0] = x;
+      }
+      __syncwarp();
+      size = 1;
+      return 0;
+    }
+    // every block's first and (if full) last key at once: the first keys find
+    // x's block b (the last one starting below x), the last keys are what the
+    // cascade passes on
+    const uint64_t first = lane < nbk ? a[(lane << 6) | hd] : KEY_MAX;
+    const uint64_t last = (lane < nbk && ((lane + 1) << 6) <= n) ? a[(lane << 6) | ((hd + 63) & 63)] : 0;
+    const int k = __popc(__ballot_sync(FULL, first < x));
+    const int b = k > 0 ? k - 1 : 0;
+    const int hb = __shfl_sync(FULL, hd, b);
+    const int cnt = min(64, n - (b << 6));
     const int s0 = (b << 6) | ((hb + lane) & 63), s1 = (b << 6) | ((hb + lane + 32) & 63);
     const uint64_t e0 = a[s0], e1 = a[s1];
+    // o = keys of block b below x (0..cnt); o == 64: x follows a full block b
+    // and is itself what b passes on
+    const int o = __popc(__ballot_sync(FULL, lane < cnt && e0 < x)) +
+                  __popc(__ballot_sync(FULL, lane + 32 < cnt && e1 < x));
+    const uint64_t v = (lane == b && o == 64) ? x : last;  // block c passes v on
+    const uint64_t vin = __shfl_up_sync(FULL, v, 1);       // lane c: block c - 1's
     const uint64_t up0 = __shfl_up_sync(FULL, e0, 1), up1 = __shfl_up_sync(FULL, e1, 1);
     const uint64_t e0_31 = __shfl_sync(FULL, e0, 31);
     __syncwarp();
     // block b: offsets k <= cnt (k < 64) take old[k] (k < o), x (k = o) or
-    // old[k - 1] (k > o); old[63] of a full block left as v above
-    if (b < nbk) {
+    // old[k - 1] (k > o); old[63] of a full block left as `last`
+    if (o < 64) {
       const int k0 = lane, k1 = lane + 32;
       const uint64_t p1 = lane == 0 ? e0_31 : up1;
       if (k0 <= cnt) a[s0] = k0 < o ? e0 : (k0 == o ? x : up0);
       if (k1 <= cnt && k1 < 64) a[s1] = k1 < o ? e1 : (k1 == o ? x : p1);
-    } else if (lane == b) {  // pos == n on a block boundary: a new block
-      hd = 0;
-      a[b << 6] = x;
     }
     // later blocks rotate by one slot and take the previous block's last key
     if (lane > b && lane < nbk) {
       hd = (hd + 63) & 63;
       a[(lane << 6) | hd] = vin;
-    } else if (lane == nbk && b < nbk && (n & 63) == 0) {  // the last block overflowed
+    } else if (lane == nbk && (n & 63) == 0) {  // the last block was full: a new block
       hd = 0;
       a[lane << 6] = vin;
     }
     __syncwarp();
     size = n + 1;
-    return pos;
+    return (b << 6) + o;
   }
   // reading R17: set the popped mark (bit 0 of a W key) of element i
   __device__ __forceinline__ void set_flag(int i, int lane) {
