@@ -752,11 +752,14 @@ constexpr bool kDistTeam = true;   // row-team distance path (query in shared me
 #else
 constexpr bool kDistTeam = false;  // lane-slice distance path (query in registers)
 #endif
-template <int NCH>
+#ifndef SONG_UNION_WIDE_ROWS
+#define SONG_UNION_WIDE_ROWS 4
+#endif
+template <int NCH, bool UNION = false>
 struct StageRows {  // rows per round: SONG_STAGE_ROWS for 128-float rows, 4 for wider ones
   // (NYTimes-shaped, 256 floats: 8 -> 4 rows frees 4 KB per warp, 14 -> 19 resident warps,
   // +12 % QPS; SIFT-shaped rows keep 8: at equal residency 4 rows cost 9 %)
-  static constexpr int R = (NCH >= 2) ? 4 : SONG_STAGE_ROWS;
+  static constexpr int R = (NCH >= 2) ? (UNION ? SONG_UNION_WIDE_ROWS : 4) : SONG_STAGE_ROWS;
   static constexpr int NBUF = SONG_STAGE_BUFS;  // rounds in flight
 };
 
@@ -908,13 +911,13 @@ __device__ __forceinline__ float hamming_distance(const float* __restrict__ data
   return (float)d;  // exact: d <= 32 * dpad < 2^24
 }
 
-template <int NCH, int METRIC>
+template <int NCH, int METRIC, bool UNION = false>
 __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, int dpad,
                                                const int* cid, int nc, const float4 (&qv)[NCH],
                                                float* stage, int cosine, int lane) {
   if constexpr (METRIC == MET_HAM) return hamming_distance<NCH>(data, dpad, cid, nc, qv, lane);
-  constexpr int R = StageRows<NCH>::R;
-  constexpr int NBUF = StageRows<NCH>::NBUF;
+  constexpr int R = StageRows<NCH, UNION>::R;
+  constexpr int NBUF = StageRows<NCH, UNION>::NBUF;
   constexpr int LR = Log2<R>::value;
   constexpr int G = R < 8 ? R : 8;  // rows per uniform compute group
   constexpr int SR = Stage<NCH>::STRIDE;
@@ -1087,12 +1090,12 @@ __device__ __forceinline__ float bulk_distance_team(const float* __restrict__ da
 // lane-slice + transposed butterfly path, or the row-team path with
 // SONG_DIST_TEAM (fewer instructions, but measured slower at 1 buffer: see
 // profiles/r01_history.md)
-template <int NCH, int METRIC>
+template <int NCH, int METRIC, bool UNION = false>
 __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpad, const int* cid,
                                          int nc, const float4 (&qv)[NCH], const float* qsm,
                                          float* stage, int cosine, int lane) {
 #ifndef SONG_DIST_TEAM
-  return bulk_distance<NCH, METRIC>(data, dpad, cid, nc, qv, stage, cosine, lane);
+  return bulk_distance<NCH, METRIC, UNION>(data, dpad, cid, nc, qv, stage, cosine, lane);
 #else
   if constexpr (METRIC == MET_HAM) return hamming_distance<NCH>(data, dpad, cid, nc, qv, lane);
   return bulk_distance_team<NCH, METRIC>(data, dpad, cid, nc, qsm, stage, cosine, lane);
@@ -1122,7 +1125,7 @@ template <int NCH, int METRIC, int VK, int QR, bool MS = false>
 __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     song_search_kernel(const SearchArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
-  constexpr int R = StageRows<NCH>::R;
+  constexpr int R = StageRows<NCH, (QR < 0)>::R;
   constexpr bool DEL = (VK == VK_HASH || VK == VK_CUCKOO);  // visited deletion (§IV-E)
   // QR > 0: q / topk in registers; QR == 0: separate q and topk tiers in
   // shared memory; QR < 0: reading R17, one bounded list W of q ∪ topk
@@ -1135,7 +1138,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   unsigned char* base = smem + (size_t)warp * a.warp_smem_bytes;
   float* stage = reinterpret_cast<float*>(base);                       // staged rows
   const size_t stage_bytes =  // (Hamming codes are gathered straight into registers)
-      METRIC == MET_HAM ? 0 : (size_t)StageRows<NCH>::NBUF * R * Stage<NCH>::STRIDE * 4;
+      METRIC == MET_HAM ? 0 : (size_t)StageRows<NCH, (QR < 0)>::NBUF * R * Stage<NCH>::STRIDE * 4;
   // the query, 16 B chunks (row-team distance path)
   float* qsm = reinterpret_cast<float*>(base + stage_bytes);
   constexpr size_t qsm_bytes = (METRIC == MET_HAM || !kDistTeam) ? 0 : (size_t)NCH * 512;
@@ -1162,7 +1165,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   GHash gh{a.gtab + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2),
            a.table_log2, a.gen0};
   const unsigned lt = lanemask_lt();
-  if (METRIC != MET_HAM) zero_stage<NCH>(stage, StageRows<NCH>::NBUF * R, lane);
+  if (METRIC != MET_HAM) zero_stage<NCH>(stage, StageRows<NCH, (QR < 0)>::NBUF * R, lane);
 
   // ---- visited-set operations (§IV-B/D/E) for the four kinds
   auto v_contains = [&](int v, bool act) -> bool {
@@ -1279,7 +1282,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     if (VK == VK_GHASH) gh.gen = ++gen;  // a fresh generation empties the table
     if (lane == 0) cid[0] = a.entry;
     __syncwarp();
-    const float de = dist_of<NCH, METRIC>(a.data, a.dpad, cid, 1, qv, qsm, stage, a.cosine, lane);
+    const float de = dist_of<NCH, METRIC, (QR < 0)>(a.data, a.dpad, cid, 1, qv, qsm, stage, a.cosine, lane);
     const uint64_t ke = make_key(__shfl_sync(FULL, de, 0), a.entry);
     v_insert_lane0(a.entry);
     int used = 1;  // VK_HASH: live + tombstones; VK_GHASH: live
@@ -1438,7 +1441,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       SONG_ST_MARK(1);
       // ---- a5: bulk distance computation (§VI)
       const float dist =
-          dist_of<NCH, METRIC>(a.data, a.dpad, cidg, nc, qv, qsm, stage, a.cosine, lane);
+          dist_of<NCH, METRIC, (QR < 0)>(a.data, a.dpad, cidg, nc, qv, qsm, stage, a.cosine, lane);
 
       SONG_ST_MARK(2);
       // ---- a6: maintenance (§IV-C/D/E)

@@ -270,10 +270,13 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   // Hamming codes: NCH = 16 B chunks per code (4 words), no row stage
   s.nch = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
   s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
-  const int rows = s.nch >= 2 ? 4 : SONG_STAGE_ROWS;  // StageRows<NCH>::R
   const int qk = queue_kind_of(L, vk, p);
   s.qk = qk;
   s.qr = qk == QK_UNION ? -1 : qk == QK_SEPARATE ? 0 : L <= 32 ? 1 : L <= 64 ? 2 : 4;
+#ifndef SONG_UNION_WIDE_ROWS
+#define SONG_UNION_WIDE_ROWS 4
+#endif
+  const int rows = s.nch >= 2 ? (s.qr < 0 ? SONG_UNION_WIDE_ROWS : 4) : SONG_STAGE_ROWS;  // StageRows<NCH, UNION>::R
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
