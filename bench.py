@@ -511,6 +511,13 @@ def run_song(args, ws, rank, local, log):
     kernel_s = sum(step_ms) / len(step_ms) / 1e3
     peak, peak_src = measured_peak_hbm()
     achieved = alg_bytes / kernel_s / 1e9
+    # replicated query batches (GIST x10) re-read the same rows from
+    # L2: the headline fraction counts the unique queries' bytes only (round-1
+    # verdict: a fraction > 1.2 from replicas is not credible); the all-query
+    # figure stays in the line as frac_all_queries
+    achieved_all = achieved
+    if reps > 1:
+        achieved = achieved_all / reps
 
     if args.profile:
         log(f"profile run: {step_ms}")
@@ -572,6 +579,9 @@ def run_song(args, ws, rank, local, log):
         "roofline": {
             "bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4),
+            **({"frac_all_queries": round(achieved_all / peak, 4),
+                "frac_note": f"frac counts the {nq // reps} unique queries' bytes; the {reps} "
+                             f"replicas of each re-read its rows from L2"} if reps > 1 else {}),
             "traffic": profiled_traffic(f"{cfg.name}:L{L_op}"),
             "kernel": kernel_name(cfg, L_op, args.visited), "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "n_dist": n_dist, "n_exp": n_exp,
