@@ -257,7 +257,9 @@ def profiled_traffic(config_key: str):
 
 
 # ------------------------------------------------------------------ workload
-GRAPH_BUILDERS = ("auto", "batched", "exact")
+GRAPH_BUILDERS = ("auto", "batched", "exact", "mips")
+GRAPH_DESC = {"batched": "song_build_graph_batched (R16)", "exact": "song_build_graph (R15)",
+              "mips": "song_graph_merge_rows of the R15 IP graph and the R16 cosine graph (R18)"}
 # song_build_graph_batched parameters of the bench's graph (override: --build-*)
 # (measured: profiles/r01u_build_sweep_sift.txt, r01t_build_sweep_nyt.txt —
 # build queue_len 128 with batches of m/4 gives SIFT1M L 32 -> 28 and NYTimes
@@ -280,8 +282,13 @@ def default_graph(cfg):
     NYTimes 768 -> 144 at recall 0.95); on the IP workload its search-built
     forward lists cap recall near 0.90, and on the 960-d GIST workload exact
     insertion needs L 28 where R16 needs 40 (profiles/r01t_bench_gist1m_exact.log),
-    so those keep exact insertion (R15)."""
-    return "exact" if cfg.metric == "ip" or cfg.dim >= 512 else "batched"
+    so those keep exact insertion (R15).  The IP workload takes the mixed graph
+    of reading R18 (the IP graph's first 8 links + the angular R16 graph:
+    recall 0.95 at L = 224 where the IP graph alone needs 1280,
+    profiles/r02u_ip_graph_probe_d.json)."""
+    if cfg.metric == "ip":
+        return "mips"
+    return "exact" if cfg.dim >= 512 else "batched"
 
 
 def build_graph_for(x, cfg, graph="auto"):
@@ -293,6 +300,9 @@ def build_graph_for(x, cfg, graph="auto"):
     if graph == "exact":
         return song.build_graph(x, cfg.degree, cfg.metric)
     b = build_params(cfg)
+    if graph == "mips":  # reading R18
+        return song.build_graph_mips(x, cfg.degree, take_ip=8, prefix=b["prefix"],
+                                     queue_len=b["queue_len"], batch_shift=b["batch_shift"])
     return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=b["prefix"],
                                     queue_len=b["queue_len"], batch_shift=b["batch_shift"])
 
@@ -566,7 +576,7 @@ def run_song(args, ws, rank, local, log):
         "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32",
         "data": f"synthetic ({data_desc(cfg)}, seeded; graph built on device by "
-                f"{'song_build_graph_batched (R16)' if graph_used == 'batched' else 'song_build_graph (R15)'})",
+                f"{GRAPH_DESC[graph_used]})",
         "config": {
             "workload": workload_desc(cfg, nq, K, L_op),
             "graph": graph_used, "n": cfg.n, "dim": d, "degree": deg, "nq_per_gpu": nq, "query_replicas": reps, "K": K, "queue_len": L_op,
@@ -887,8 +897,7 @@ def run_reference(args, ws, rank, local, log):
         "ms_per_step": round(1e3 * sum(times) / len(times), 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f64",
         "data": f"synthetic ({data_desc(cfg)}, seeded; graph built by a child process with "
-                f"{'song_build_graph_batched (R16)' if graph_used == 'batched' else 'song_build_graph (R15)'}, "
-                f"loaded from a file: this process never maps libsong.so)",
+                f"{GRAPH_DESC[graph_used]}, loaded from a file: this process never maps libsong.so)",
         "impl": "reference",
         "config": {"workload": workload_desc(cfg, cfg.nq * reps, cfg.K, L_op), "graph": graph_used,
                    "queue_len": L_op, "recall_sweep": sweep},

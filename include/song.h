@@ -406,6 +406,20 @@ int song_build_graph_from_forward(const float* vectors, int64_t n, int32_t dim,
  * instrumentation; cycles_out is zeroed). */
 int song_stage_cycles(song_index* idx, uint64_t* cycles_out, int32_t reset);
 
+/* Reading R18 (graphs for the inner-product metric): row v of out = the first
+ * `take_first` ids of first[v], then the ids of second[v], then the rest of
+ * first[v] — each id once (its first occurrence), -1 skipped, truncated to
+ * `degree`, -1 padded.  With first = the IP graph (song_build_graph, SONG_IP)
+ * and second = the angular graph (song_build_graph_batched, SONG_COSINE) this
+ * keeps each vertex's best inner-product links and fills the row with
+ * direction-preserving ones, which the IP search navigates far better than
+ * either graph alone (R18).
+ *   first, second, out  DEVICE [n][degree] int32 (out may not alias the inputs)
+ * Asynchronous on stream.  Errors: SONG_EINVAL (NULL, n < 1, degree < 1,
+ * take_first outside [0, degree]), SONG_EUNSUPPORTED (degree > 32). */
+int song_graph_merge_rows(const int32_t* first, const int32_t* second, int64_t n,
+                          int32_t degree, int32_t take_first, int32_t* out, void* stream);
+
 /* Thread-local message of the last failing call ("" if none). */
 const char* song_last_error(void);
 

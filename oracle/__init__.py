@@ -367,3 +367,22 @@ def merge_shards(ids_per_shard, dists_per_shard, K: int):
             out_i[r, j] = i
             out_d[r, j] = d
     return out_i, out_d
+
+
+def merge_graph_rows(first, second, take_first: int):
+    """Reading R18, written out: row v = first[v][:take], then second[v], then
+    first[v][take:], each id once (first occurrence), -1 skipped, truncated to
+    the degree, -1 padded."""
+    first = np.asarray(first)
+    second = np.asarray(second)
+    n, D = first.shape
+    out = np.full((n, D), -1, np.int32)
+    for v in range(n):
+        seq = list(first[v][:take_first]) + list(second[v]) + list(first[v][take_first:])
+        kept = []
+        for i in seq:
+            if i >= 0 and i not in kept:
+                kept.append(int(i))
+        kept = kept[:D]
+        out[v, :len(kept)] = kept
+    return out

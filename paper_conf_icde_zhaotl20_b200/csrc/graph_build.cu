@@ -270,7 +270,66 @@ __global__ void keys_from_results_kernel(const int32_t* __restrict__ ids,
   }
 }
 
+// reading R18: row v = the first `take` ids of first[v], then the ids of
+// second[v], then the rest of first[v] — each id once (first occurrence),
+// -1 skipped, truncated to degree, -1 padded.  One warp per row, lane j =
+// slot j of each input row.
+__global__ void merge_rows_kernel(const int32_t* __restrict__ first,
+                                  const int32_t* __restrict__ second, int64_t n, int degree,
+                                  int take, int32_t* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  unsigned lt;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+  for (int64_t v = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const int a = lane < degree ? first[v * degree + lane] : -1;
+    const int b = lane < degree ? second[v * degree + lane] : -1;
+    // the candidate sequence: a[0..take), b[0..D), a[take..D)
+    int nk = 0;        // ids kept so far (warp-uniform)
+    int mine = -1;     // lane j < nk: the j-th kept id
+    auto take_from = [&](int id, bool in) {
+      bool keep = in && id >= 0;
+      // first occurrence inside this group
+      const unsigned grp = __match_any_sync(0xffffffffu, keep ? id : -1 - lane);
+      keep = keep && (grp & lt) == 0;
+      // not kept before
+      for (int j = 0; j < nk; ++j) {  // (the shuffle outside the &&: every lane calls it)
+        const int kj = __shfl_sync(0xffffffffu, mine, j);
+        keep = keep && kj != id;
+      }
+      const unsigned m = __ballot_sync(0xffffffffu, keep);
+      const int pos = nk + __popc(m & lt);
+      // lane pos receives id: every lane with keep sends to lane pos
+      for (unsigned mm = m; mm; mm &= mm - 1) {
+        const int src = __ffs(mm) - 1;
+        const int idv = __shfl_sync(0xffffffffu, id, src);
+        const int p = nk + __popc(m & ((1u << src) - 1));
+        if (lane == p) mine = idv;
+      }
+      nk = min(32, nk + __popc(m));
+    };
+    take_from(a, lane < take);
+    take_from(b, true);
+    take_from(a, lane >= take);
+    if (lane < degree) out[v * degree + lane] = lane < nk ? mine : -1;
+  }
+}
+
 }  // namespace
+
+extern "C" int song_graph_merge_rows(const int32_t* first, const int32_t* second, int64_t n,
+                                     int32_t degree, int32_t take_first, int32_t* out,
+                                     void* stream) {
+  if (!first || !second || !out) return fail(SONG_EINVAL, "NULL argument");
+  if (n < 1 || degree < 1) return fail(SONG_EINVAL, "n and degree must be >= 1");
+  if (degree > SONG_MAX_DEGREE) return fail(SONG_EUNSUPPORTED, "degree %d > %d", degree, SONG_MAX_DEGREE);
+  if (take_first < 0 || take_first > degree)
+    return fail(SONG_EINVAL, "take_first %d outside [0, degree]", take_first);
+  const int blocks = (int)std::min<int64_t>((n + 7) / 8, 148 * 64);
+  merge_rows_kernel<<<blocks, 256, 0, (cudaStream_t)stream>>>(first, second, n, degree, take_first, out);
+  G_TRY(cudaGetLastError());
+  return SONG_OK;
+}
 
 extern "C" int song_build_graph(const float* vectors, int64_t n, int32_t dim, song_metric metric,
                                 int32_t degree, int32_t* adjacency_out, void* stream) {

@@ -34,7 +34,8 @@ EXPORTED = ["song_default_params", "song_index_create", "song_index_create_devic
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
             "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward",
-            "song_search_plan_get", "song_stage_cycles", "song_merge_topk_peers"]
+            "song_search_plan_get", "song_stage_cycles", "song_merge_topk_peers",
+            "song_graph_merge_rows"]
 
 
 class SongError(RuntimeError):
@@ -105,6 +106,7 @@ def lib():
         L.song_search_plan_get.argtypes = [ctypes.POINTER(SearchParams), i32, i32,
                                            ctypes.POINTER(SearchPlan)]
         L.song_stage_cycles.argtypes = [P, P, i32]
+        L.song_graph_merge_rows.argtypes = [P, P, i64, i32, i32, P, P]
         L.song_merge_topk_peers.argtypes = [P, P, P, i32, i32, i64, i32, i32, ctypes.c_uint32,
                                             P, P, P]
         L.song_last_error.restype = ctypes.c_char_p
@@ -117,7 +119,7 @@ def lib():
                      "song_index_create_codes", "song_index_create_rp",
                      "song_search_codes_ex", "song_build_graph", "song_build_graph_batched",
                      "song_build_graph_from_forward", "song_search_plan_get",
-                     "song_stage_cycles", "song_merge_topk_peers"):
+                     "song_stage_cycles", "song_merge_topk_peers", "song_graph_merge_rows"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -348,6 +350,32 @@ def merge_topk(ids, dists, K: int):
                                  G, nq, kin, K, ctypes.c_void_p(oi.data_ptr()),
                                  ctypes.c_void_p(od.data_ptr()), _stream_ptr(ids.device)))
     return oi, od
+
+
+def merge_graph_rows(first, second, take_first: int):
+    """song_graph_merge_rows (reading R18): CUDA int32 [n, degree] graphs ->
+    the merged rows (first `take_first` of `first`, then `second`, then the
+    rest of `first`; ids once, -1 padded)."""
+    torch = _torch()
+    a = first.to(torch.int32).contiguous()
+    b = second.to(device=a.device, dtype=torch.int32).contiguous()
+    assert a.shape == b.shape
+    out = torch.empty_like(a)
+    _check(lib().song_graph_merge_rows(ctypes.c_void_p(a.data_ptr()), ctypes.c_void_p(b.data_ptr()),
+                                       a.shape[0], a.shape[1], int(take_first),
+                                       ctypes.c_void_p(out.data_ptr()), _stream_ptr(a.device)))
+    return out
+
+
+def build_graph_mips(vectors, degree: int = 32, take_ip: int = 8, prefix: int = 1 << 16,
+                     queue_len: int = 128, batch_shift: int = 2):
+    """Reading R18: the inner-product graph = each vertex's first `take_ip`
+    links of the IP graph (song_build_graph, exact insertion) filled with the
+    angular graph's (song_build_graph_batched, cosine)."""
+    ip = build_graph(vectors, degree, "ip")
+    cos = build_graph_batched(vectors, degree, "cosine", prefix=prefix, queue_len=queue_len,
+                              batch_shift=batch_shift)
+    return merge_graph_rows(ip, cos, take_ip)
 
 
 def merge_topk_peers(ids_ptrs, dists_ptrs, nq: int, kin: int, K: int, out=None,

@@ -35,7 +35,7 @@ def test_graph_choice_and_builder_params_per_config():
     assert bench.default_graph(CONFIGS["sift1m"]) == "batched"
     assert bench.default_graph(CONFIGS["nytimes256"]) == "batched"
     assert bench.default_graph(CONFIGS["gist1m"]) == "exact"
-    assert bench.default_graph(CONFIGS["glove200"]) == "exact"
+    assert bench.default_graph(CONFIGS["glove200"]) == "mips"
     for name in ("sift1m", "nytimes256"):
         b = bench.build_params(CONFIGS[name])
         assert b == bench.BUILD

@@ -229,3 +229,22 @@ def test_tensor_core_path_only_when_exact(monkeypatch):
     auto = gbuild(x, 16)
     monkeypatch.setenv("SONG_GRAPH_PATH", "simt")
     np.testing.assert_array_equal(auto, gbuild(x, 16))
+
+
+@pytest.mark.parametrize("take", [0, 1, 8, 31, 32])
+def test_merge_graph_rows_bit_exact(take):
+    """song_graph_merge_rows (reading R18) against the oracle's definition, on
+    rows with padding, repeats inside a row and ids shared by both rows."""
+    rng = np.random.default_rng(take)
+    n, D = 3000, 32
+    a = rng.integers(-1, 200, (n, D)).astype(np.int32)
+    b = rng.integers(-1, 200, (n, D)).astype(np.int32)
+    s = song()
+    got = s.merge_graph_rows(torch.as_tensor(a, device="cuda"), torch.as_tensor(b, device="cuda"),
+                             take).cpu().numpy()
+    np.testing.assert_array_equal(got, oracle.merge_graph_rows(a, b, take))
+    for D2 in (7, 16):  # degrees below 32
+        a2, b2 = a[:, :D2].copy(), b[:, :D2].copy()
+        got = s.merge_graph_rows(torch.as_tensor(a2, device="cuda"),
+                                 torch.as_tensor(b2, device="cuda"), min(take, D2)).cpu().numpy()
+        np.testing.assert_array_equal(got, oracle.merge_graph_rows(a2, b2, min(take, D2)))

@@ -167,3 +167,15 @@ def test_batched_graph_is_valid_and_searchable():
     ids, _, _, _ = oracle.search(x, adj, q, 10, 64)
     truth, _ = oracle.bruteforce(x, q, 10)
     assert oracle.recall(ids, truth) > 0.9
+
+
+def test_merge_graph_rows_definition():
+    """Reading R18 on hand-worked rows: the first `take` of the IP row, then the
+    angular row, then the rest of the IP row; ids once, -1 skipped, truncated."""
+    first = np.array([[1, 2, 3, -1], [0, 2, 2, 5], [-1, -1, -1, -1]], np.int32)
+    second = np.array([[3, 4, 5, 1], [5, 6, -1, 0], [7, -1, 8, 7]], np.int32)
+    got = oracle.merge_graph_rows(first, second, 2)
+    np.testing.assert_array_equal(got, [[1, 2, 3, 4], [0, 2, 5, 6], [7, 8, -1, -1]])
+    # take 0 = the second graph first; take D = the first graph first
+    np.testing.assert_array_equal(oracle.merge_graph_rows(first, second, 0)[0], [3, 4, 5, 1])
+    np.testing.assert_array_equal(oracle.merge_graph_rows(first, second, 4)[1], [0, 2, 5, 6])
