@@ -257,9 +257,9 @@ def profiled_traffic(config_key: str):
 
 
 # ------------------------------------------------------------------ workload
-GRAPH_BUILDERS = ("auto", "batched", "exact", "mips")
+GRAPH_BUILDERS = ("auto", "batched", "exact", "mixed")
 GRAPH_DESC = {"batched": "song_build_graph_batched (R16)", "exact": "song_build_graph (R15)",
-              "mips": "song_graph_merge_rows of the R15 IP graph and the R16 cosine graph (R18)"}
+              "mixed": "song_graph_merge_rows of two device-built graphs (R18, bench.MIXED)"}
 # song_build_graph_batched parameters of the bench's graph (override: --build-*)
 # (measured: profiles/r01u_build_sweep_sift.txt, r01t_build_sweep_nyt.txt —
 # build queue_len 128 with batches of m/4 gives SIFT1M L 32 -> 28 and NYTimes
@@ -276,18 +276,25 @@ def build_params(cfg):
     return p
 
 
+# reading R18 per workload: (graph A, graph B, links kept from A), measured with
+# tools/mix_graph_probe.py / ip_graph_probe.py (profiles/r02u_*, r02y_*): the
+# L reaching recall 0.95 drops SIFT 28 -> 20, NYTimes 144 -> 80, GIST 28 -> 24,
+# GloVe-IP 1280 -> 224
+MIXED = {"sift1m": ("batched:l2", "exact:l2", 16),
+         "nytimes256": ("batched:cosine", "exact:cosine", 24),
+         "gist1m": ("exact:l2", "batched:l2", 24),
+         "glove200": ("exact:ip", "batched:cosine", 8)}
+
+
 def default_graph(cfg):
-    """Measured per workload: batched insertion (R16) gives the
-    SIFT / cosine workloads better graphs than exact insertion (SIFT1M L 48 -> 32,
-    NYTimes 768 -> 144 at recall 0.95); on the IP workload its search-built
-    forward lists cap recall near 0.90, and on the 960-d GIST workload exact
-    insertion needs L 28 where R16 needs 40 (profiles/r01t_bench_gist1m_exact.log),
-    so those keep exact insertion (R15).  The IP workload takes the mixed graph
-    of reading R18 (the IP graph's first 8 links + the angular R16 graph:
-    recall 0.95 at L = 224 where the IP graph alone needs 1280,
-    profiles/r02u_ip_graph_probe_d.json)."""
+    """Measured per workload (reading R18): the mixed graph where
+    one is defined for the workload (R15 exact insertion is O(n^2), so not at
+    100M rows), else batched insertion (R16) — the IP workload's R16 lists
+    plateau at recall 0.90 and 960-d GIST prefers R15 (exact)."""
+    if cfg.name in MIXED and cfg.K == 10:  # (measured at K = 10; K = 100 runs at L = K, where
+        return "mixed"                        # R16 alone expands less: 5.50 M vs 5.36 M QPS)
     if cfg.metric == "ip":
-        return "mips"
+        return "exact"
     return "exact" if cfg.dim >= 512 else "batched"
 
 
@@ -300,9 +307,16 @@ def build_graph_for(x, cfg, graph="auto"):
     if graph == "exact":
         return song.build_graph(x, cfg.degree, cfg.metric)
     b = build_params(cfg)
-    if graph == "mips":  # reading R18
-        return song.build_graph_mips(x, cfg.degree, take_ip=8, prefix=b["prefix"],
-                                     queue_len=b["queue_len"], batch_shift=b["batch_shift"])
+    if graph == "mixed":  # reading R18: the first `take` links of A, then B's
+        sa, sb, take = MIXED[cfg.name]
+
+        def one(spec):
+            kind, metric = spec.split(":")
+            if kind == "exact":
+                return song.build_graph(x, cfg.degree, metric)
+            return song.build_graph_batched(x, cfg.degree, metric, prefix=b["prefix"],
+                                            queue_len=b["queue_len"], batch_shift=b["batch_shift"])
+        return song.merge_graph_rows(one(sa), one(sb), take)
     return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=b["prefix"],
                                     queue_len=b["queue_len"], batch_shift=b["batch_shift"])
 

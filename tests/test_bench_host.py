@@ -32,10 +32,13 @@ def test_gpu_local_cpus_without_gpu_is_empty():
 
 def test_graph_choice_and_builder_params_per_config():
     from workloads.synth import CONFIGS
-    assert bench.default_graph(CONFIGS["sift1m"]) == "batched"
-    assert bench.default_graph(CONFIGS["nytimes256"]) == "batched"
-    assert bench.default_graph(CONFIGS["gist1m"]) == "exact"
-    assert bench.default_graph(CONFIGS["glove200"]) == "mips"
+    for name in ("sift1m", "nytimes256", "gist1m", "glove200"):
+        assert bench.default_graph(CONFIGS[name]) == "mixed"
+        a, b, take = bench.MIXED[name]
+        assert 0 < take < CONFIGS[name].degree
+        assert {a.split(":")[0], b.split(":")[0]} == {"exact", "batched"}
+    assert bench.MIXED["glove200"][1] == "batched:cosine"  # the angular fill of the IP graph
+    assert bench.default_graph(CONFIGS["scaleout100m"]) == "batched"  # R15 is O(n^2)
     for name in ("sift1m", "nytimes256"):
         b = bench.build_params(CONFIGS[name])
         assert b == bench.BUILD
