@@ -78,11 +78,17 @@ def sharded(a, x, q, truth, song, bench, torch, np):
             shard_ms.append(e0.elapsed_time(e1))
             ids_g.append(i)
             d_g.append(d)
+        # the fused gather + merge kernel of the multi-GPU path (song_merge_topk_peers),
+        # here reading the G shards' result buffers through a pointer table
+        ptr = lambda ts: torch.tensor([t.data_ptr() for t in ts], dtype=torch.int64, device=dev)  # noqa: E731
+        pi, pd = ptr(ids_g), ptr(d_g)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        mi, _ = song.merge_topk(torch.stack(ids_g), torch.stack(d_g), 10)
+        mi, _ = song.merge_topk_peers(pi, pd, q.shape[0], 10, 10)
         e1.record()
         torch.cuda.synchronize()
+        mi2, _ = song.merge_topk(torch.stack(ids_g), torch.stack(d_g), 10)
+        assert torch.equal(mi, mi2)
         r = bench.recall_t(mi, torch.as_tensor(truth, device=dev))
         step_ms = max(shard_ms) + e0.elapsed_time(e1)
         out["sweep"].append({"L": L, "recall": round(r, 4), "max_shard_ms": round(max(shard_ms), 4),
@@ -110,7 +116,7 @@ def main():
     ap.add_argument("--shards", type=int, default=0,
                     help="also run dataset sharding (P:471, SURVEY §8(e)(ii)): G shards with "
                          "their own graphs, every query searched on every shard, merged by "
-                         "song_merge_topk; emulated on this GPU one shard at a time")
+                         "song_merge_topk_peers; emulated on this GPU one shard at a time")
     ap.add_argument("--out", default="gpurun_out/scaleout.json")
     a = ap.parse_args()
     import numpy as np
