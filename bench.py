@@ -540,8 +540,9 @@ def run_song(args, ws, rank, local, log):
     # verdict: a fraction > 1.2 from replicas is not credible); the all-query
     # figure stays in the line as frac_all_queries
     achieved_all = achieved
-    if reps > 1:
-        achieved = achieved_all / reps
+    traffic = profiled_traffic(f"{cfg.name}:L{L_op}")
+    if reps > 1:  # per DRAM byte when a capture is committed, else per unique query
+        achieved = traffic / kernel_s / 1e9 if traffic else achieved_all / reps
 
     if args.profile:
         log(f"profile run: {step_ms}")
@@ -604,9 +605,12 @@ def run_song(args, ws, rank, local, log):
             "bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4),
             **({"frac_all_queries": round(achieved_all / peak, 4),
-                "frac_note": f"frac counts the {nq // reps} unique queries' bytes; the {reps} "
-                             f"replicas of each re-read its rows from L2"} if reps > 1 else {}),
-            "traffic": profiled_traffic(f"{cfg.name}:L{L_op}"),
+                "frac_note": (f"frac = ncu DRAM bytes per launch (profiles/traffic.json) / kernel "
+                              f"time: the {reps} replicas of each of the {nq // reps} unique queries "
+                              f"re-read its rows from L2" if traffic else
+                              f"frac counts the {nq // reps} unique queries' bytes; the {reps} "
+                              f"replicas of each re-read its rows from L2")} if reps > 1 else {}),
+            "traffic": traffic,
             "kernel": kernel_name(cfg, L_op, args.visited), "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "n_dist": n_dist, "n_exp": n_exp,
             "kernel_ms": round(kernel_s * 1e3, 4),
