@@ -98,6 +98,8 @@ def parse():
                          "(weak scaling); dataset: the rows are split over the ranks, each with "
                          "its own graph, rank 0's batch is broadcast and the per-shard top-K "
                          "merged by the fused symmetric-memory kernel (P:471; strong scaling)")
+    ap.add_argument("--schedule", default="auto", choices=["auto", "batch", "outlier_first"],
+                    help="song_search_params.schedule: ticket order of the batch's queries")
     ap.add_argument("--queue-kind", default="auto", choices=["auto", "separate", "union"],
                     help="song_search_params.queue_kind (results never depend on it)")
     ap.add_argument("--warps-per-block", type=int, default=0)
@@ -464,7 +466,8 @@ def run_song(args, ws, rank, local, log):
     def params(L):
         return song.Params(K=cfg.K, queue_len=L, visited=args.visited,
                            warps_per_block=args.warps_per_block, blocks_per_sm=args.blocks_per_sm,
-                           visited_cap=args.visited_cap, queue_kind=args.queue_kind)
+                           visited_cap=args.visited_cap, queue_kind=args.queue_kind,
+                           schedule=args.schedule)
 
     # ---- operating point: smallest grid queue_len with recall@10 >= target
     sweep = []

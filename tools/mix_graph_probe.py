@@ -29,6 +29,8 @@ def main():
     ap.add_argument("--b", default="exact:l2")
     ap.add_argument("--take", default="32,24,16,8")
     ap.add_argument("--L", default="16,20,24,28,32,40,48")
+    ap.add_argument("--bq", type=int, default=128, help="R16 build queue_len")
+    ap.add_argument("--bs", type=int, default=2, help="R16 batch_shift")
     ap.add_argument("--out", default="")
     a = ap.parse_args()
     import torch
@@ -38,8 +40,8 @@ def main():
     log = lambda m: print(f"[probe] {m}", file=sys.stderr, flush=True)  # noqa: E731
     x, q0 = make_data(cfg, device="cuda")
     truth = bench.ground_truth(x, q0, cfg.K, cfg.metric)
-    ga, gb = build(a.a, x, cfg, song), build(a.b, x, cfg, song)
-    res = {"config": cfg.name, "a": a.a, "b": a.b, "recall": {}, "qps": {}}
+    ga, gb = build(a.a, x, cfg, song, a.bq, a.bs), build(a.b, x, cfg, song, a.bq, a.bs)
+    res = {"config": cfg.name, "a": a.a, "b": a.b, "bq": a.bq, "bs": a.bs, "recall": {}, "qps": {}}
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     for k in map(int, a.take.split(",")):
         adj = ga if k >= cfg.degree else song.merge_graph_rows(ga, gb, k)
