@@ -110,6 +110,10 @@ def main():
     ap.add_argument("--build-queue-len", type=int, default=128)
     ap.add_argument("--batch-shift", type=int, default=2)
     ap.add_argument("--compare-exact", action="store_true")
+    ap.add_argument("--mix", default="",
+                    help="reading R18 at scale: 'queue_len:shift:take' builds a second R16 graph "
+                         "with those builder parameters and searches the row merge (the first "
+                         "`take` links of the first graph, then the second's)")
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--parity-sample", type=int, default=0,
                     help="queries the oracle recomputes one by one at the operating point")
@@ -154,6 +158,19 @@ def main():
     torch.cuda.synchronize()
     res["build_s"] = round(time.time() - t0, 1)
     print("built", res["build_s"], "s", flush=True)
+    if a.mix:
+        bq, bs, take = (int(v) for v in a.mix.split(":"))
+        t0 = time.time()
+        g2 = song.build_graph_batched(x, 32, "l2", prefix=a.prefix, queue_len=bq, batch_shift=bs)
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+        graphs["mixed"] = song.merge_graph_rows(graphs["batched"], g2, take)
+        del g2
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+        res["build_mixed_s"] = round(time.time() - t0, 1)
+        res["mix"] = {"second_queue_len": bq, "second_batch_shift": bs, "take": take}
+        print("mixed built", res["build_mixed_s"], "s", flush=True)
     if a.compare_exact:
         t0 = time.time()
         graphs["exact"] = song.build_graph(x, 32, "l2")

@@ -15,7 +15,11 @@ import bench  # noqa: E402
 
 
 def build(spec, x, cfg, song, bq=128, bs=2):
-    kind, metric = spec.split(":")
+    """spec = kind:metric[:build_queue_len:batch_shift]"""
+    parts = spec.split(":")
+    kind, metric = parts[0], parts[1]
+    if len(parts) == 4:
+        bq, bs = int(parts[2]), int(parts[3])
     if kind == "exact":
         return song.build_graph(x, cfg.degree, metric)
     return song.build_graph_batched(x, cfg.degree, metric, prefix=1 << 16, queue_len=bq,
