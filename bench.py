@@ -278,14 +278,16 @@ def build_params(cfg):
     return p
 
 
-# reading R18 per workload: (graph A, graph B, links kept from A), measured with
-# tools/mix_graph_probe.py / ip_graph_probe.py (profiles/r02u_*, r02y_*): the
-# L reaching recall 0.95 drops SIFT 28 -> 20, NYTimes 144 -> 80, GIST 28 -> 24,
-# GloVe-IP 1280 -> 224
-MIXED = {"sift1m": ("batched:l2", "exact:l2", 16),
-         "nytimes256": ("batched:cosine", "exact:cosine", 24),
-         "gist1m": ("exact:l2", "batched:l2", 24),
-         "glove200": ("exact:ip", "batched:cosine", 8)}
+# reading R18 per workload: graph = the first builder's, then merged row by row
+# with each further builder's (`song_graph_merge_rows`, keeping the first `take`
+# links of the rows so far); spec = kind:metric[:build_queue_len:batch_shift].
+# Measured with tools/mix_graph_probe.py, ip_graph_probe.py, mix3_probe.py
+# (profiles/r02u_*, r02y_*, r02mix3_*): the L reaching recall 0.95 drops SIFT
+# 28 -> 16, NYTimes 144 -> 56, GIST 28 -> 24, GloVe-IP 1280 -> 160
+MIXED = {"sift1m": ["batched:l2:128:2", ("batched:l2:64:1", 20), ("exact:l2", 28)],
+         "nytimes256": ["batched:cosine:128:2", ("batched:cosine:64:1", 20), ("exact:cosine", 28)],
+         "gist1m": ["exact:l2", ("batched:l2:128:2", 24)],
+         "glove200": ["exact:ip", ("batched:cosine:128:2", 8), ("batched:cosine:64:1", 20)]}
 
 
 def default_graph(cfg):
@@ -309,16 +311,22 @@ def build_graph_for(x, cfg, graph="auto"):
     if graph == "exact":
         return song.build_graph(x, cfg.degree, cfg.metric)
     b = build_params(cfg)
-    if graph == "mixed":  # reading R18: the first `take` links of A, then B's
-        sa, sb, take = MIXED[cfg.name]
+    if graph == "mixed":  # reading R18: row merges of device-built graphs
+        chain = MIXED[cfg.name]
 
         def one(spec):
-            kind, metric = spec.split(":")
+            parts = spec.split(":")
+            kind, metric = parts[0], parts[1]
             if kind == "exact":
                 return song.build_graph(x, cfg.degree, metric)
+            bq, bs = (int(parts[2]), int(parts[3])) if len(parts) == 4 else (b["queue_len"],
+                                                                           b["batch_shift"])
             return song.build_graph_batched(x, cfg.degree, metric, prefix=b["prefix"],
-                                            queue_len=b["queue_len"], batch_shift=b["batch_shift"])
-        return song.merge_graph_rows(one(sa), one(sb), take)
+                                            queue_len=bq, batch_shift=bs)
+        adj = one(chain[0])
+        for spec, take in chain[1:]:
+            adj = song.merge_graph_rows(adj, one(spec), take)
+        return adj
     return song.build_graph_batched(x, cfg.degree, cfg.metric, prefix=b["prefix"],
                                     queue_len=b["queue_len"], batch_shift=b["batch_shift"])
 

@@ -34,10 +34,13 @@ def test_graph_choice_and_builder_params_per_config():
     from workloads.synth import CONFIGS
     for name in ("sift1m", "nytimes256", "gist1m", "glove200"):
         assert bench.default_graph(CONFIGS[name]) == "mixed"
-        a, b, take = bench.MIXED[name]
-        assert 0 < take < CONFIGS[name].degree
-        assert {a.split(":")[0], b.split(":")[0]} == {"exact", "batched"}
-    assert bench.MIXED["glove200"][1] == "batched:cosine"  # the angular fill of the IP graph
+        chain = bench.MIXED[name]
+        assert isinstance(chain[0], str) and len(chain) >= 2
+        for spec, take in chain[1:]:
+            assert 0 < take < CONFIGS[name].degree
+            assert spec.split(":")[0] in ("exact", "batched")
+    assert bench.MIXED["glove200"][0] == "exact:ip"  # the IP graph's links first ...
+    assert bench.MIXED["glove200"][1][0].startswith("batched:cosine")  # ... then angular ones
     assert bench.default_graph(CONFIGS["scaleout100m"]) == "batched"  # R15 is O(n^2)
     for name in ("sift1m", "nytimes256"):
         b = bench.build_params(CONFIGS[name])
