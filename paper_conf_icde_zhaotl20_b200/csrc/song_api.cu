@@ -207,13 +207,26 @@ struct Shape {
 #ifndef SONG_HASH_UNION_DEN
 #define SONG_HASH_UNION_DEN 3
 #endif
-int hash_log2_slots(int L, bool uni = false) {
+// wide rows (NCH >= 2: > 128 floats, a 4 KB+ stage per warp) take F = 4 for
+// L <= 64: shared memory, not recomputation, is their limit (NYTimes-shaped
+// L = 56: 5.94 M -> 6.39 M QPS; SIFT-shaped rows keep 8: 19.6 M vs 18.4 M,
+// profiles/r03hf_*)
+#ifndef SONG_HASH_FACTOR_WIDEROW
+#define SONG_HASH_FACTOR_WIDEROW 4
+#endif
+int nch_of(int dpad, bool hamming) {
+  int n = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
+  return n <= 1 ? 1 : n <= 2 ? 2 : n <= 4 ? 4 : 8;
+}
+
+int hash_log2_slots(int L, bool uni = false, int nch = 1) {
   if (uni)
     return next_pow2_log2((SONG_HASH_UNION_NUM * (L + 32ll) + SONG_HASH_UNION_DEN - 1) /
                           SONG_HASH_UNION_DEN);
   const long long live = 2ll * L + 32;
   if (L > 128) return next_pow2_log2((SONG_HASH_BIG_NUM * live + SONG_HASH_BIG_DEN - 1) / SONG_HASH_BIG_DEN);
-  const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE : SONG_HASH_FACTOR;
+  const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE
+                     : nch >= 2 ? SONG_HASH_FACTOR_WIDEROW : SONG_HASH_FACTOR;
   return next_pow2_log2(F * live);
 }
 
@@ -246,7 +259,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     tbytes = (4 << s.table_log2) * 2;
   } else if (queue_kind_of(L, vk, p) == QK_UNION) {
     // R17: live keys <= |W| + 32 new ones <= L + 32; lazy by default
-    s.table_log2 = hash_log2_slots(L, true);
+    s.table_log2 = hash_log2_slots(L, true, nch_of(dpad, hamming));
     s.lazy = p->visited_cap >= 0;
     s.rebuild_at = s.lazy && p->visited_cap > 0 ? p->visited_cap : (3 << s.table_log2) / 4;
     tbytes = (1 << s.table_log2) * 4;
@@ -257,7 +270,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     // probe per operation); shared-memory queues (L > 128) get >= 2x and
     // rebuild at 3/4 to bound shared memory.
     const bool big = L > 128;
-    s.table_log2 = hash_log2_slots(L);
+    s.table_log2 = hash_log2_slots(L, false, nch_of(dpad, hamming));
     s.rebuild_at = big ? (3 << s.table_log2) / 4 : (SONG_HASH_REBUILD_NUM << s.table_log2) / 16;
     // lazy deletion (R14): visited holds up to C live ids, no tombstones
     s.lazy = p->visited_cap >= 0 && p->steps <= 1;
@@ -268,8 +281,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   }
   // float rows: NCH = 16 B chunks per lane (128 floats per chunk row);
   // Hamming codes: NCH = 16 B chunks per code (4 words), no row stage
-  s.nch = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
-  s.nch = s.nch <= 1 ? 1 : s.nch <= 2 ? 2 : s.nch <= 4 ? 4 : 8;
+  s.nch = nch_of(dpad, hamming);
   const int qk = queue_kind_of(L, vk, p);
   s.qk = qk;
   s.qr = qk == QK_UNION ? -1 : qk == QK_SEPARATE ? 0 : L <= 32 ? 1 : L <= 64 ? 2 : 4;
@@ -340,14 +352,7 @@ int check_params_common(const song_search_params* p, int metric) {
     return fail(SONG_EINVAL, "unknown queue_kind %d", p->queue_kind);
   if (p->queue_kind == SONG_QUEUE_UNION && (p->visited != SONG_VISITED_HASH || p->steps > 1))
     return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH and steps <= 1");
-  if (p->visited_cap > 0 && p->visited == SONG_VISITED_HASH) {
-    const bool uni = queue_kind_of(p->queue_len, song::VK_HASH, p) == QK_UNION;
-    const int slots = 1 << hash_log2_slots(p->queue_len, uni);
-    const int lo = uni ? p->queue_len + 32 : 2 * p->queue_len + 32;
-    if (p->visited_cap < lo || p->visited_cap > 3 * (slots / 4))
-      return fail(SONG_EINVAL, "visited_cap %d outside [%d, 3/4 of %d slots]", p->visited_cap,
-                  lo, slots);
-  }
+
   if (p->schedule < SONG_SCHEDULE_AUTO || p->schedule > SONG_SCHEDULE_OUTLIER_FIRST)
     return fail(SONG_EINVAL, "unknown schedule %d", p->schedule);
   if (p->steps > SONG_MAX_STEPS)
@@ -366,8 +371,24 @@ int check_params_common(const song_search_params* p, int metric) {
   return SONG_OK;
 }
 
+// an explicit lazy capacity must lie in [live bound, 3/4 of the table]
+int check_cap(const song_search_params* p, int dpad, int metric) {
+  if (p->visited_cap > 0 && p->visited == SONG_VISITED_HASH) {
+    const bool uni = queue_kind_of(p->queue_len, song::VK_HASH, p) == QK_UNION;
+    const int slots =
+        1 << hash_log2_slots(p->queue_len, uni, nch_of(dpad, metric == SONG_HAMMING));
+    const int lo = uni ? p->queue_len + 32 : 2 * p->queue_len + 32;
+    if (p->visited_cap < lo || p->visited_cap > 3 * (slots / 4))
+      return fail(SONG_EINVAL, "visited_cap %d outside [%d, 3/4 of %d slots]", p->visited_cap,
+                  lo, slots);
+  }
+  return SONG_OK;
+}
+
 int check_params(const song_index* ix, const song_search_params* p) {
   int rc = check_params_common(p, ix->metric);
+  if (rc) return rc;
+  rc = check_cap(p, ix->dpad, ix->metric);
   if (rc) return rc;
   if (p->entry < 0 || p->entry >= ix->n) return fail(SONG_EINVAL, "entry %d out of range", p->entry);
   return SONG_OK;
@@ -809,6 +830,8 @@ int song_search_plan_get(const song_search_params* p, int32_t dim, int32_t metri
   if (metric == SONG_HAMMING && dim * 32 > SONG_MAX_CODE_BITS)
     return fail(SONG_EUNSUPPORTED, "%d code words > %d bits", dim, SONG_MAX_CODE_BITS);
   int rc = check_params_common(p, metric);
+  if (rc) return rc;
+  rc = check_cap(p, dpad_of(dim, metric), metric);
   if (rc) return rc;
   Shape sh;
   rc = plan_shape(p, dpad_of(dim, metric), metric, &sh);

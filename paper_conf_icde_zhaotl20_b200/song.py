@@ -314,6 +314,12 @@ class SongIndex:
             ctypes.c_void_p(ctr.data_ptr() if ctr is not None else 0), _stream_ptr(q.device)))
         return (ids, dists, ctr) if counters else (ids, dists)
 
+    def plan(self, params: "Params") -> "SearchPlan":
+        """song_search_plan_get for this index (its dimension and metric)."""
+        info = self.info()
+        dim = info.dim_padded if self.metric == "hamming" else info.dim
+        return plan(params, dim, self.metric)
+
     def stage_cycles(self, reset: bool = True):
         """song_stage_cycles (SONG_STAGE_TIMING builds): SM cycles per stage
         [pop/topk, locate, distance, maintenance] summed over warps."""

@@ -88,7 +88,7 @@ def test_full_size_sampled_parity(name, K, sample):
     rng = np.random.default_rng(1)
     pick = np.sort(rng.choice(q.shape[0], sample, replace=False))
     o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()[pick], K, L_op,
-                      metric=oracle.METRICS[cfg.metric], nthreads=8, **oracle_kw("hash", L_op))
+                      metric=oracle.METRICS[cfg.metric], nthreads=8, **oracle_kw("hash", L_op, idx=idx))
     g = (gi[pick], gd[pick], gc[pick])
     if cfg.kind == "sift":
         assert_exact(g, o)

@@ -45,7 +45,7 @@ def song_plan_cap(L, dim, metric):
     return s.default_visited_cap(L, dim, metric)
 
 
-def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0, queue_kind="auto"):
+def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0, queue_kind="auto", idx=None):
     """The oracle mode matching a GPU search, read from the library's plan
     (song_search_plan_get): the hash's deletion schedule is lazy (reading
     R14) unless visited_cap = -1 or steps > 1 (eager), and queues above 128
@@ -53,8 +53,9 @@ def oracle_kw(visited, L, steps=1, visited_cap=0, log2=0, queue_kind="auto"):
     from paper_conf_icde_zhaotl20_b200 import song as s
     kw = dict(flags=ORACLE_FLAGS[visited], bloom_bits=bloom_bits_for(L, log2, visited))
     if visited == "hash":
-        pl = s.plan(s.Params(K=1, queue_len=L, steps=steps, visited_cap=visited_cap,
-                             queue_kind=queue_kind), 128)
+        prm = s.Params(K=1, queue_len=L, steps=steps, visited_cap=visited_cap,
+                       queue_kind=queue_kind)
+        pl = idx.plan(prm) if idx is not None else s.plan(prm, 128)
         flags = oracle.OPTIMIZED
         if pl.visited_cap > 0:
             flags |= oracle.LAZY
@@ -116,7 +117,7 @@ def test_fig1_toy_on_gpu(visited):
     ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited)
     assert [int(x) + 1 for x in ids[0]] == result
     o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
-                      **oracle_kw(visited, 3))
+                      **oracle_kw(visited, 3, idx=idx))
     assert_exact((ids, d, c), o)
     if visited == "hash":
         # the paper's literal (eager) deletion: Fig. 4(c), 12 distances, 4 expansions
@@ -145,7 +146,7 @@ def test_tiny_parity(tiny, L, visited):
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q, cfg.K, L, visited)
-    o = oracle.search(x, adj, q, cfg.K, L, **oracle_kw(visited, L))
+    o = oracle.search(x, adj, q, cfg.K, L, **oracle_kw(visited, L, idx=idx))
     assert_close(g, o, truth, scale=float(np.abs(o[1]).max()))
 
 
@@ -169,7 +170,7 @@ def test_sift_integer_bit_exact(sift100k, L, visited, warps):
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q.cpu().numpy(), cfg.K, L, visited, warps_per_block=warps)
     o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), cfg.K, L,
-                      **oracle_kw(visited, L),
+                      **oracle_kw(visited, L, idx=idx),
                       nthreads=8)
     assert_exact(g, o)
 
@@ -265,12 +266,12 @@ def test_edges_exact(dim, L, K):
     idx = s.SongIndex(x, adj)
     for visited in ALL_VISITED:
         g = gpu_search(idx, q, K, L, visited)
-        o = oracle.search(x, adj, q, K, L, **oracle_kw(visited, L))
+        o = oracle.search(x, adj, q, K, L, **oracle_kw(visited, L, idx=idx))
         assert_exact(g, o)
     for qk in ("union", "separate"):  # every queue kind at every L (R17 / §IV-C)
         for cap in (0, -1):
             g = gpu_search(idx, q, K, L, "hash", queue_kind=qk, visited_cap=cap)
-            o = oracle.search(x, adj, q, K, L, **oracle_kw("hash", L, visited_cap=cap, queue_kind=qk))
+            o = oracle.search(x, adj, q, K, L, **oracle_kw("hash", L, visited_cap=cap, queue_kind=qk, idx=idx))
             assert_exact(g, o)
 
 
@@ -286,7 +287,7 @@ def test_union_queue_bit_exact(sift100k, L, cap):
     idx = s.SongIndex(x, adj)
     xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()[:200]
     g = gpu_search(idx, qn, cfg.K, L, "hash", visited_cap=cap)
-    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap))
+    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap, idx=idx))
     assert o is not None and s.plan(s.Params(K=1, queue_len=L), 128).queue_kind == 2
     assert_exact(g, o)
     sep = gpu_search(idx, qn, cfg.K, L, "hash", queue_kind="separate")
@@ -314,14 +315,14 @@ def test_large_queue_len_max():
     s = song()
     idx = s.SongIndex(x, adj)
     g = gpu_search(idx, q[:16], 100, 2048)
-    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048))
+    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, idx=idx))
     assert_exact(g, o)
     g = gpu_search(idx, q[:16], 100, 2048, visited_cap=-1)  # eager deletion
-    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, visited_cap=-1))
+    o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, visited_cap=-1, idx=idx))
     assert_exact(g, o)
     for qk in ("separate", "union"):  # both shared-memory queue kinds at the maximum
         g = gpu_search(idx, q[:16], 100, 2048, queue_kind=qk)
-        o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, queue_kind=qk))
+        o = oracle.search(x, adj, q[:16], 100, 2048, **oracle_kw("hash", 2048, queue_kind=qk, idx=idx))
         assert_exact(g, o)
 
 
@@ -439,7 +440,7 @@ def test_fused_peer_merge_over_symmetric_memory(sift100k, tmp_path):
             torch.cuda.synchronize()
         assert si._merger.epoch == 2
         oi, od, _, _ = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy(), K, L,
-                                     nthreads=8, **oracle_kw("hash", L))
+                                     nthreads=8, **oracle_kw("hash", L, idx=si.index))
         ei, ed = oracle.merge_shards([oi], [od], K)
         np.testing.assert_array_equal(fi.cpu().numpy(), ei)
         np.testing.assert_array_equal(fd.cpu().numpy(), ed)
@@ -458,9 +459,9 @@ def test_deletion_schedules_exact(sift100k, L, cap):
     idx = s.SongIndex(x, adj)
     xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()
     g = gpu_search(idx, qn, cfg.K, L, "hash", visited_cap=cap)
-    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap))
+    o = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=cap, idx=idx))
     assert_exact(g, o)
-    eager = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=-1))
+    eager = oracle.search(xn, an, qn, cfg.K, L, nthreads=8, **oracle_kw("hash", L, visited_cap=-1, idx=idx))
     np.testing.assert_array_equal(g[0], eager[0])  # the schedule never changes results
     np.testing.assert_array_equal(g[1], eager[1])
     if cap != -1:
@@ -485,7 +486,7 @@ def test_sift1m_full_size_sampled_parity():
     pick = np.sort(rng.choice(cfg.nq, 300, replace=False))
     xn, an = x.cpu().numpy(), adj.cpu().numpy()
     o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 48, nthreads=8,
-                      **oracle_kw("hash", 48))
+                      **oracle_kw("hash", 48, idx=idx))
     assert_exact((ids.cpu().numpy()[pick], d.cpu().numpy()[pick], c.cpu().numpy()[pick]), o)
     # properties that hold for every query at any size: sorted, unique, valid ids
     ii, dd = ids.cpu().numpy(), d.cpu().numpy()
@@ -538,7 +539,7 @@ def test_schedule_never_changes_results(name, L):
             np.testing.assert_array_equal(a, b)
     pick = np.arange(0, 6000, 40)
     o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()[pick], cfg.K, L,
-                      metric=oracle.METRICS[cfg.metric], nthreads=8, **oracle_kw("hash", L))
+                      metric=oracle.METRICS[cfg.metric], nthreads=8, **oracle_kw("hash", L, idx=idx))
     g = tuple(r[pick] for r in res["outlier_first"])
     if cfg.kind == "sift":
         assert_exact(g, o)
@@ -561,7 +562,7 @@ def test_max_dim_exact(dim):
     idx = s.SongIndex(x, adj)
     for visited in ("hash", "bloom"):
         g = gpu_search(idx, q, 10, 40, visited)
-        o = oracle.search(x, adj, q, 10, 40, **oracle_kw(visited, 40))
+        o = oracle.search(x, adj, q, 10, 40, **oracle_kw(visited, 40, idx=idx))
         assert_exact(g, o)
     idx.close()
 
@@ -574,9 +575,38 @@ def test_single_vertex_and_isolated_entry():
     idx = s.SongIndex(x, np.full((1, 4), -1, np.int32))
     g = gpu_search(idx, np.zeros((2, 2), np.float32), 3, 4)
     o = oracle.search(x, np.full((1, 4), -1, np.int32), np.zeros((2, 2), np.float32), 3, 4,
-                      **oracle_kw("hash", 4))
+                      **oracle_kw("hash", 4, idx=idx))
     assert_exact(g, o)
     assert (g[0][:, 0] == 0).all() and (g[0][:, 1:] == -1).all()
     assert (g[1][:, 0] == 25.0).all() and np.isinf(g[1][:, 1:]).all()
     assert (g[2] == [[1, 1]]).all()
     idx.close()
+
+
+def test_stage_cycles_only_in_instrumented_builds():
+    """song_stage_cycles: the product library is built without
+    SONG_STAGE_TIMING and says so (SONG_EUNSUPPORTED, zeroed output)."""
+    x, adj, q = small_random(n=300, dim=8)
+    s = song()
+    idx = s.SongIndex(x, adj)
+    gpu_search(idx, q, 10, 16)
+    with pytest.raises(s.SongError) as e:
+        idx.stage_cycles()
+    assert e.value.code == -4
+
+
+def test_search_plan_matches_the_launch():
+    """The plan (song_search_plan_get, host-only) is what the search runs: the
+    lazy capacity it reports reproduces the GPU's counters in the oracle for a
+    narrow (NCH 1) and a wide (NCH 2) row, where the table sizes differ."""
+    s = song()
+    for dim in (16, 200):
+        x, adj, q = small_random(n=2000, dim=dim, deg=16)
+        idx = s.SongIndex(x, adj)
+        for L in (32, 64, 100, 200):
+            pl = idx.plan(s.Params(K=10, queue_len=L))
+            assert pl.visited_cap > 0
+            g = gpu_search(idx, q, 10, L)
+            flags = oracle.OPTIMIZED_LAZY | (oracle.UNION if pl.queue_kind == 2 else 0)
+            o = oracle.search(x, adj, q, 10, L, flags=flags, lazy_cap=pl.visited_cap)
+            assert_exact(g, o)

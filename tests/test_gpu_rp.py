@@ -80,7 +80,7 @@ def test_hamming_search_bit_exact(mnist, bits, L, visited):
     torch.cuda.synchronize()
     idx.last_status()
     from test_gpu_parity import oracle_kw
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, K, L, nthreads=8, **oracle_kw(visited, L))
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, K, L, nthreads=8, **oracle_kw(visited, L, idx=idx))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
@@ -109,7 +109,7 @@ def test_rp_index_end_to_end(mnist, monkeypatch, chunk_rows):
     codes = oracle.rp_encode(x, R, nthreads=8)
     qc = oracle.rp_encode(q, R, nthreads=8)
     from test_gpu_parity import oracle_kw
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 1, 64, nthreads=8, **oracle_kw("hash", 64))
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 1, 64, nthreads=8, **oracle_kw("hash", 64, idx=idx))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)
@@ -160,7 +160,7 @@ def test_code_footprint_is_table4s(mnist, bits):
                                  s.Params(K=5, queue_len=40), counters=True)
     torch.cuda.synchronize()
     from test_gpu_parity import oracle_kw
-    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 5, 40, **oracle_kw("hash", 40))
+    oi, od, oc, _ = oracle.search_codes(codes, adj, qc, 5, 40, **oracle_kw("hash", 40, idx=idx))
     np.testing.assert_array_equal(ids.cpu().numpy(), oi)
     np.testing.assert_array_equal(d.cpu().numpy(), od)
     np.testing.assert_array_equal(c.cpu().numpy().astype(np.int64), oc)

@@ -45,7 +45,7 @@ def test_scaleout_100m_sampled_parity():
     del adj
     xn = x.cpu().numpy()
     o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 64, nthreads=16,
-                      **oracle_kw("hash", 64))
+                      **oracle_kw("hash", 64, idx=idx))
     assert_exact((gi[pick], gd[pick], gc[pick]), o)
     # every row of the graph: ids in range, no self loop, no repeats (sampled rows)
     rows = an[np.random.default_rng(0).choice(cfg.n, 20_000, replace=False)]
