@@ -594,6 +594,28 @@ def run_song(args, ws, rank, local, log):
         if i >= 3:
             h2d_s.append(time.perf_counter() - t)
     del qd
+    # ---- end to end as a serving loop: `steps` batches of the same shape
+    # streamed through song_search_pipelined (each batch's HtoD, search and
+    # DtoH inside the timed call; two batches in flight, the next batch's
+    # kernel filling the SMs the previous one's persistent grid releases)
+    nb = max(args.steps, 2)
+    qp = torch.empty((nb,) + tuple(q.shape), dtype=torch.float32, pin_memory=True)
+    qp.copy_(qh.unsqueeze(0).expand_as(qp))
+    ip = torch.empty((nb, nq, K), dtype=torch.int32, pin_memory=True)
+    dp = torch.empty((nb, nq, K), dtype=torch.float32, pin_memory=True)
+    nw = max(2, min(nb, args.warmup))
+    for _ in range(2):  # untimed: the second lane, buffers and events are made on first use
+        idx.search_pipelined_into(qp[:nw], p, ip[:nw], dp[:nw])
+    flush.zero_()
+    torch.cuda.synchronize()
+    barrier(ws)
+    t = time.perf_counter()
+    idx.search_pipelined_into(qp, p, ip, dp)
+    pipe_s = allreduce_max(time.perf_counter() - t, ws)
+    pipe_value = ws * nq * nb / pipe_s
+    pipe_ok = bool((ip.numpy() == out[0].cpu().numpy()[None]).all()
+                   and (dp.numpy() == out[1].cpu().numpy()[None]).all())
+    del qp, ip, dp
     os.sched_setaffinity(0, all_cpus)  # the CPU baseline uses every core
 
     result = {
@@ -627,18 +649,24 @@ def run_song(args, ws, rank, local, log):
             "kernel_ms": round(kernel_s * 1e3, 4),
             "kernel_ms_note": "whole step on the launching stream: search kernel + outlier-first scheduling kernels (conservative for the search kernel alone)",
         },
-        "e2e": {"value": round(e2e_value, 1), "unit": "queries/s",
+        "e2e": {"value": round(pipe_value, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(qh.numel() * 4),
                 "d2h_bytes_per_step": int(ih.numel() * 4 + dh.numel() * 4),
-                "host_results_match_device": host_ok,
+                "mode": (f"song_search_pipelined: {nb} host batches of {nq} queries in one "
+                         f"timed call (wall clock, max over ranks); each batch's HtoD from "
+                         f"pinned memory, search and DtoH inside; two batches in flight; L2 "
+                         f"flushed before the call, not between its batches"),
+                "ms_per_step": round(pipe_s / nb * 1e3, 4),
+                "host_results_match_device": bool(host_ok and pipe_ok),
                 "host_cpus": f"{len(near)} GPU-local cores (NUMA node of the GPU)" if near
                              else f"{len(all_cpus)} cores (GPU locality unknown)",
-                # wall-clock per call (value above = steps / their sum): host
-                # jitter on the box shows up as max >> median
-                "h2d_ms_median": round(sorted(h2d_s)[len(h2d_s) // 2] * 1e3, 4),
-                "ms_per_step": {"min": round(min(e2e_s) * 1e3, 4),
-                                "median": round(sorted(e2e_s)[len(e2e_s) // 2] * 1e3, 4),
-                                "max": round(max(e2e_s) * 1e3, 4)}},
+                # one blocking song_search per batch (HtoD, kernel, DtoH
+                # serialised), L2 flushed before each call; wall clock per call
+                "per_call": {"value": round(e2e_value, 1), "api": "song_search",
+                             "h2d_ms_median": round(sorted(h2d_s)[len(h2d_s) // 2] * 1e3, 4),
+                             "ms_per_step": {"min": round(min(e2e_s) * 1e3, 4),
+                                             "median": round(sorted(e2e_s)[len(e2e_s) // 2] * 1e3, 4),
+                                             "max": round(max(e2e_s) * 1e3, 4)}}},
         "clocks": clk.summary(),
         # per step: the search kernel, plus the two outlier-first scheduling
         # kernels (order keys + scatter) when the batch outnumbers the resident

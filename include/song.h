@@ -242,6 +242,26 @@ int song_index_get_info(const song_index* idx, song_index_info* info);
 int song_search(song_index* idx, const float* queries, int64_t nq, int32_t K,
                 int32_t queue_len, int32_t* ids_out, float* dists_out);
 
+/* Search a STREAM of nbatch query batches held in HOST memory (the batched
+ * throughput setting of §VIII, with Fig. 10's HtoD / kernel / DtoH per
+ * batch); blocking.
+ *   queries   [nbatch][nq][dim] fp32 host (dim = song_index_info.dim);
+ *   ids_out   [nbatch][nq][K] int32 host; dists_out [nbatch][nq][K] fp32 host.
+ * Batch b's results are exactly those of song_search_ex(params) on batch b
+ * alone (every query is searched independently; the ticket order never
+ * changes results).  The call keeps two batches in flight on two device
+ * buffer sets with their own work counters: the HtoD copy of batch b + 1 and
+ * the DtoH copy of batch b - 1 run on copy streams under the search of batch
+ * b, and batch b + 1's search kernel takes the SMs batch b's persistent grid
+ * releases in its tail (two compute streams).  Page-locked host buffers
+ * (cudaHostAlloc, torch pin_memory) let the copies overlap; pageable ones
+ * give the same results with serialised copies.  Ordered after any search
+ * previously enqueued on the index.  Errors: as song_search (SONG_EINVAL also
+ * for nbatch < 1); the sticky status covers every batch. */
+int song_search_pipelined(song_index* idx, const song_search_params* params,
+                          const float* queries, int64_t nbatch, int64_t nq,
+                          int32_t* ids_out, float* dists_out);
+
 /* Search with DEVICE buffers on a caller stream; asynchronous (returns after
  * enqueueing).  counters_out, if not NULL, receives [nq][2] int32
  * (distance computations, expansions) per query — the algorithmic work that

@@ -129,6 +129,18 @@ int alloc_index(song_index* ix, int64_t n, int32_t dim, int32_t degree, song_met
 
 void free_index(song_index* ix) {
   if (!ix) return;
+  if (ix->twin) free_index(ix->twin);
+  if (ix->is_twin) {  // the rows, graph, centroid and R belong to the owner
+    ix->d_data = nullptr;
+    ix->d_adj = nullptr;
+    ix->d_centroid = nullptr;
+    ix->d_R = nullptr;
+  }
+  if (ix->h2d) cudaStreamDestroy(ix->h2d);
+  if (ix->d2h) cudaStreamDestroy(ix->d2h);
+  if (ix->ev_h2d) cudaEventDestroy(ix->ev_h2d);
+  if (ix->ev_done) cudaEventDestroy(ix->ev_done);
+  if (ix->ev_out) cudaEventDestroy(ix->ev_out);
   cudaFree(ix->d_data);
   cudaFree(ix->d_adj);
   cudaFree(ix->d_ticket);
@@ -1012,19 +1024,11 @@ int song_index_last_status(song_index* ix) {
   return status_code(st);
 }
 
-int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int32_t queue_len,
-                int32_t* ids_out, float* dists_out) {
-  if (!ix || !queries || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
-  if (nq < 1) return fail(SONG_EINVAL, "nq must be >= 1");
-  song_search_params p;
-  song_default_params(&p, K, queue_len);
-  int rc = check_params(ix, &p);
-  if (rc) return rc;
-  if (ix->metric == SONG_HAMMING && !ix->d_R)
-    return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
-  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
-  const size_t qbytes = (size_t)nq * qdim * sizeof(float);
-  const size_t obytes = (size_t)nq * K * sizeof(int32_t);
+}  // extern "C"
+
+namespace {
+// device buffers of the host-buffer entry points (grown, never shrunk)
+int ensure_io(song_index* ix, size_t qbytes, size_t obytes) {
   if (qbytes > ix->cap_q) {
     cudaFree(ix->d_q);
     ix->d_q = nullptr;
@@ -1042,6 +1046,63 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
     CUDA_TRY(cudaMalloc(&ix->d_dists, obytes));
     ix->cap_out = obytes;
   }
+  return SONG_OK;
+}
+
+int make_events(song_index* ix) {
+  if (!ix->ev_h2d) CUDA_TRY(cudaEventCreateWithFlags(&ix->ev_h2d, cudaEventDisableTiming));
+  if (!ix->ev_done) CUDA_TRY(cudaEventCreateWithFlags(&ix->ev_done, cudaEventDisableTiming));
+  if (!ix->ev_out) CUDA_TRY(cudaEventCreateWithFlags(&ix->ev_out, cudaEventDisableTiming));
+  return SONG_OK;
+}
+
+// the second lane of song_search_pipelined: shares the owner's rows, graph,
+// centroid and R (read-only in every kernel), owns the rest
+int ensure_twin(song_index* ix) {
+  if (ix->twin) return SONG_OK;
+  song_index* t = new song_index();
+  t->is_twin = true;
+  t->device = ix->device;
+  t->num_sms = ix->num_sms;
+  t->n = ix->n;
+  t->dim = ix->dim;
+  t->dpad = ix->dpad;
+  t->degree = ix->degree;
+  t->metric = ix->metric;
+  t->d_data = ix->d_data;
+  t->d_adj = ix->d_adj;
+  t->dedup = ix->dedup;
+  t->code_bits = ix->code_bits;
+  t->rp_dim = ix->rp_dim;
+  t->d_R = ix->d_R;
+  t->d_centroid = ix->d_centroid;
+  ix->twin = t;  // freed with the owner from here on
+  CUDA_TRY(cudaMalloc(&t->d_ticket, sizeof(unsigned)));
+  CUDA_TRY(cudaMalloc(&t->d_status, sizeof(int)));
+  CUDA_TRY(cudaMemset(t->d_status, 0, sizeof(int)));
+  CUDA_TRY(cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking));
+  t->last_stream = t->stream;
+  return SONG_OK;
+}
+}  // namespace
+
+extern "C" {
+
+int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int32_t queue_len,
+                int32_t* ids_out, float* dists_out) {
+  if (!ix || !queries || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (nq < 1) return fail(SONG_EINVAL, "nq must be >= 1");
+  song_search_params p;
+  song_default_params(&p, K, queue_len);
+  int rc = check_params(ix, &p);
+  if (rc) return rc;
+  if (ix->metric == SONG_HAMMING && !ix->d_R)
+    return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
+  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
+  const size_t qbytes = (size_t)nq * qdim * sizeof(float);
+  const size_t obytes = (size_t)nq * K * sizeof(int32_t);
+  rc = ensure_io(ix, qbytes, obytes);
+  if (rc) return rc;
   cudaStream_t st = ix->stream;
   rc = order_after_last(ix, st);
   if (rc) return rc;
@@ -1062,6 +1123,81 @@ int song_search(song_index* ix, const float* queries, int64_t nq, int32_t K, int
   CUDA_TRY(cudaMemsetAsync(ix->d_status, 0, sizeof(int), st));
   CUDA_TRY(cudaStreamSynchronize(st));
   return status_code(*ix->h_status);
+}
+
+int song_search_pipelined(song_index* ix, const song_search_params* p, const float* queries,
+                          int64_t nbatch, int64_t nq, int32_t* ids_out, float* dists_out) {
+  if (!ix || !p || !queries || !ids_out || !dists_out) return fail(SONG_EINVAL, "NULL argument");
+  if (nbatch < 1 || nq < 1) return fail(SONG_EINVAL, "nbatch and nq must be >= 1");
+  if (nq > 0x7fffffffll) return fail(SONG_EUNSUPPORTED, "nq must fit int32");
+  if (ix->is_twin) return fail(SONG_EINVAL, "not an index handle");
+  int rc = check_params(ix, p);
+  if (rc) return rc;
+  if (ix->metric == SONG_HAMMING && !ix->d_R)
+    return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
+  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
+  const size_t qbytes = (size_t)nq * qdim * sizeof(float);
+  const size_t obytes = (size_t)nq * p->K * sizeof(int32_t);
+  const int nl = nbatch > 1 ? 2 : 1;
+  if (nl == 2) {
+    rc = ensure_twin(ix);
+    if (rc) return rc;
+  }
+  song_index* lane[2] = {ix, ix->twin};
+  if (!ix->h2d) CUDA_TRY(cudaStreamCreateWithFlags(&ix->h2d, cudaStreamNonBlocking));
+  if (!ix->d2h) CUDA_TRY(cudaStreamCreateWithFlags(&ix->d2h, cudaStreamNonBlocking));
+  for (int l = 0; l < nl; ++l) {
+    rc = ensure_io(lane[l], qbytes, obytes);
+    if (!rc) rc = make_events(lane[l]);
+    if (rc) return rc;
+    // after every search enqueued earlier on the index (any stream)
+    if (ix->last_done) CUDA_TRY(cudaStreamWaitEvent(lane[l]->stream, ix->last_done, 0));
+    lane[l]->last_stream = lane[l]->stream;
+  }
+  // the copy streams too: a lane's buffers may still be read by an earlier call
+  if (ix->last_done) {
+    CUDA_TRY(cudaStreamWaitEvent(ix->h2d, ix->last_done, 0));
+    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, ix->last_done, 0));
+  }
+  const char* qh = reinterpret_cast<const char*>(queries);
+  char* ih = reinterpret_cast<char*>(ids_out);
+  char* dh = reinterpret_cast<char*>(dists_out);
+  for (int64_t b = 0; b < nbatch; ++b) {
+    song_index* L = lane[b % nl];
+    cudaStream_t st = L->stream;
+    // HtoD of batch b once the lane's previous search (b - nl) has read d_q
+    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(ix->h2d, L->ev_done, 0));
+    CUDA_TRY(cudaMemcpyAsync(L->d_q, qh + b * qbytes, qbytes, cudaMemcpyHostToDevice, ix->h2d));
+    CUDA_TRY(cudaEventRecord(L->ev_h2d, ix->h2d));
+    CUDA_TRY(cudaStreamWaitEvent(st, L->ev_h2d, 0));
+    // the lane's outputs once the DtoH of batch b - nl has read them
+    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(st, L->ev_out, 0));
+    const float* dq = L->d_q;
+    if (ix->metric == SONG_HAMMING) {
+      rc = encode_queries(L, L->d_q, nq, st);
+      if (rc) return rc;
+      dq = reinterpret_cast<const float*>(L->d_qcodes);
+    }
+    rc = enqueue_search(L, p, dq, nq, L->d_ids, L->d_dists, nullptr, st);
+    if (rc) return rc;
+    CUDA_TRY(cudaEventRecord(L->ev_done, st));
+    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, L->ev_done, 0));
+    CUDA_TRY(cudaMemcpyAsync(ih + b * obytes, L->d_ids, obytes, cudaMemcpyDeviceToHost, ix->d2h));
+    CUDA_TRY(cudaMemcpyAsync(dh + b * obytes, L->d_dists, obytes, cudaMemcpyDeviceToHost, ix->d2h));
+    CUDA_TRY(cudaEventRecord(L->ev_out, ix->d2h));
+  }
+  // the last DtoH waits for the last search, which follows every earlier one
+  // on its lane; the other lane's last search precedes its own DtoH on d2h
+  CUDA_TRY(cudaStreamSynchronize(ix->d2h));
+  int st_all = 0;
+  for (int l = 0; l < nl; ++l) {
+    int s = 0;
+    CUDA_TRY(cudaMemcpy(&s, lane[l]->d_status, sizeof s, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemset(lane[l]->d_status, 0, sizeof s));
+    st_all |= s;
+  }
+  ix->last_stream = ix->stream;
+  return status_code(st_all);
 }
 
 int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,

@@ -47,6 +47,13 @@ struct song_index {
   size_t cap_order = 0;
   int* h_status = nullptr;             // pinned: song_search's status read-back
   unsigned long long* d_stage = nullptr;  // SONG_STAGE_TIMING builds: [4] cycles
+  // song_search_pipelined: a second lane (its own work counter, status, order
+  // scratch, buffers and compute stream; the rows, graph, centroid and R are
+  // this index's), copy streams, and per-lane events
+  song_index* twin = nullptr;
+  bool is_twin = false;
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t ev_h2d = nullptr, ev_done = nullptr, ev_out = nullptr;
 };
 
 namespace song {

@@ -30,7 +30,7 @@ STATUS = {0: "SONG_OK", -1: "SONG_EINVAL", -2: "SONG_ENOMEM", -3: "SONG_ECUDA",
           -4: "SONG_EUNSUPPORTED", -5: "SONG_EITERCAP"}
 
 EXPORTED = ["song_default_params", "song_index_create", "song_index_create_device",
-            "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex",
+            "song_index_destroy", "song_index_get_info", "song_search", "song_search_ex", "song_search_pipelined",
             "song_index_last_status", "song_merge_topk", "song_last_error", "song_version",
             "song_rp_encode", "song_index_create_codes", "song_index_create_rp",
             "song_search_codes_ex", "song_build_graph", "song_build_graph_batched", "song_build_graph_from_forward",
@@ -94,6 +94,7 @@ def lib():
         L.song_index_get_info.argtypes = [P, ctypes.POINTER(IndexInfo)]
         L.song_search.argtypes = [P, P, i64, i32, i32, P, P]
         L.song_search_ex.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, P, P, P, P]
+        L.song_search_pipelined.argtypes = [P, ctypes.POINTER(SearchParams), P, i64, i64, P, P]
         L.song_index_last_status.argtypes = [P]
         L.song_merge_topk.argtypes = [P, P, i32, i64, i32, i32, P, P, P]
         L.song_rp_encode.argtypes = [P, i64, i32, P, i32, P, P]
@@ -288,6 +289,27 @@ class SongIndex:
             return ctypes.c_void_p(x.data_ptr() if hasattr(x, "data_ptr") else
                                    x.ctypes.data)
         _check(lib().song_search(self._h, ptr(q), q.shape[0], K, queue_len, ptr(ids), ptr(dists)))
+
+    def search_pipelined_into(self, q, params: "Params", ids, dists):
+        """song_search_pipelined: q [nbatch, nq, dim] HOST (numpy or pinned CPU
+        tensor), ids / dists [nbatch, nq, K] HOST; blocking."""
+        def ptr(x):
+            return ctypes.c_void_p(x.data_ptr() if hasattr(x, "data_ptr") else
+                                   x.ctypes.data)
+        if len(q.shape) != 3 or tuple(ids.shape) != (q.shape[0], q.shape[1], params.K) \
+                or tuple(dists.shape) != tuple(ids.shape):
+            raise ValueError("q [nbatch, nq, dim], ids / dists [nbatch, nq, K]")
+        pc = params.to_c()
+        _check(lib().song_search_pipelined(self._h, ctypes.byref(pc), ptr(q), q.shape[0],
+                                           q.shape[1], ptr(ids), ptr(dists)))
+
+    def search_pipelined(self, queries: np.ndarray, params: "Params"):
+        """song_search_pipelined on host batches [nbatch, nq, dim] -> (ids, dists)."""
+        q = np.ascontiguousarray(queries, np.float32)
+        ids = np.empty((q.shape[0], q.shape[1], params.K), np.int32)
+        dists = np.empty(ids.shape, np.float32)
+        self.search_pipelined_into(q, params, ids, dists)
+        return ids, dists
 
     def search(self, queries, K: int = 10, queue_len: int = 64, params: Optional[Params] = None,
                counters: bool = False, out=None):

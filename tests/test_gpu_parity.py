@@ -224,6 +224,66 @@ def test_host_and_device_entry_points_agree(sift100k):
     np.testing.assert_array_equal(qd, g[1])
 
 
+@pytest.mark.parametrize("L,visited,nbatch", [(64, "hash", 5), (16, "hash", 1), (48, "hashtable", 4),
+                                             (1024, "hash", 3), (48, "cuckoo", 2)])
+def test_pipelined_batches_match_single_searches(sift100k, L, visited, nbatch):
+    """song_search_pipelined (two lanes in flight, copy streams, the next
+    batch's kernel in the previous one's tail) returns, batch by batch, what
+    song_search_ex returns for that batch alone — and the oracle's answer."""
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    qn = q.cpu().numpy()
+    nq = qn.shape[0] // nbatch
+    qb = np.ascontiguousarray(qn[:nq * nbatch].reshape(nbatch, nq, -1))
+    p = s.Params(K=cfg.K, queue_len=L, visited=visited)
+    ids, dists = idx.search_pipelined(qb, p)
+    for b in range(nbatch):
+        g = gpu_search(idx, qb[b], cfg.K, L, visited)
+        np.testing.assert_array_equal(ids[b], g[0])
+        np.testing.assert_array_equal(dists[b], g[1])
+    o = oracle.search(x.cpu().numpy(), adj.cpu().numpy(), qb.reshape(nq * nbatch, -1), cfg.K, L,
+                      nthreads=8, **oracle_kw(visited, L, idx=idx))
+    np.testing.assert_array_equal(ids.reshape(nq * nbatch, -1), o[0])
+    np.testing.assert_array_equal(dists.reshape(nq * nbatch, -1), o[1])
+    # the call is repeatable (lanes and events are reused) and ordered after
+    # a device search enqueued just before it on torch's stream
+    idx.search(q, params=p)
+    ids2, dists2 = idx.search_pipelined(qb, p)
+    np.testing.assert_array_equal(ids2, ids)
+
+
+def test_pipelined_large_batches_overlap(sift100k):
+    """Batches larger than the resident grid (outlier-first order, tails
+    overlapping the next batch's kernel) on pinned host buffers."""
+    cfg, x, _, adj = sift100k
+    s = song()
+    _, qbig = make_data(cfg, device="cpu", n=1000, nq=12_000)
+    qb = torch.empty((3, 4000, cfg.dim), dtype=torch.float32, pin_memory=True)
+    qb.copy_(qbig.reshape(3, 4000, -1))
+    ih = torch.empty((3, 4000, cfg.K), dtype=torch.int32, pin_memory=True)
+    dh = torch.empty((3, 4000, cfg.K), dtype=torch.float32, pin_memory=True)
+    idx = s.SongIndex(x, adj)
+    p = s.Params(K=cfg.K, queue_len=32)
+    idx.search_pipelined_into(qb, p, ih, dh)
+    for b in range(3):
+        g = gpu_search(idx, qb[b].numpy(), cfg.K, 32)
+        np.testing.assert_array_equal(ih[b].numpy(), g[0])
+        np.testing.assert_array_equal(dh[b].numpy(), g[1])
+
+
+def test_pipelined_argument_errors(sift100k):
+    cfg, x, q, adj = sift100k
+    s = song()
+    idx = s.SongIndex(x, adj)
+    qb = np.zeros((2, 4, cfg.dim), np.float32)
+    with pytest.raises(s.SongError, match="EINVAL"):
+        idx.search_pipelined(qb, s.Params(K=10, queue_len=5))
+    qb[1, 2, 3] = np.nan  # a non-finite query in the second batch: sticky status
+    with pytest.raises(s.SongError, match="EINVAL"):
+        idx.search_pipelined(qb, s.Params(K=10, queue_len=16))
+
+
 # ------------------------------------------------ other metrics / dimensions
 @pytest.mark.parametrize("name,n", [("glove200", 30_000), ("nytimes256", 30_000),
                                     ("gist1m", 20_000)])

@@ -38,6 +38,7 @@ def test_scaleout_100m_sampled_parity():
     ids, d, c = idx.search(q, params=s.Params(K=cfg.K, queue_len=64), counters=True)
     torch.cuda.synchronize()
     idx.last_status()
+    okw = oracle_kw("hash", 64, idx=idx)  # the plan of this index, read before close
     idx.close()
     pick = np.arange(0, cfg.nq, cfg.nq // 100)
     gi, gd, gc = ids.cpu().numpy(), d.cpu().numpy(), c.cpu().numpy()
@@ -45,7 +46,7 @@ def test_scaleout_100m_sampled_parity():
     del adj
     xn = x.cpu().numpy()
     o = oracle.search(xn, an, q.cpu().numpy()[pick], cfg.K, 64, nthreads=16,
-                      **oracle_kw("hash", 64, idx=idx))
+                      **okw)
     assert_exact((gi[pick], gd[pick], gc[pick]), o)
     # every row of the graph: ids in range, no self loop, no repeats (sampled rows)
     rows = an[np.random.default_rng(0).choice(cfg.n, 20_000, replace=False)]
