@@ -384,13 +384,18 @@ def recall_t(ids, truth):
     return float(hit.any(2).float().sum(1).div(truth.shape[1]).mean())
 
 
-def kernel_name(cfg, L, visited):
-    dpad = (cfg.dim + 3) // 4 * 4
-    nch = (dpad + 127) // 128
-    nch = 1 if nch <= 1 else 2 if nch <= 2 else 4 if nch <= 4 else 8
-    qr = 1 if L <= 32 else 2 if L <= 64 else 4 if L <= 128 else 0
+def kernel_name(cfg, plan, visited):
+    """The search kernel's template instance for a plan (song_search_plan_get):
+    QR = 1/2/4 separate register q / topk, 0 shared-memory tiers, 8 + r the
+    bounded union W (reading R17) in r registers, -1/-2 W in tiers."""
     met = "L2" if cfg.metric == "l2" else "DOT"
-    return f"song_search_kernel<NCH={nch},{met},{visited.upper()},QR={qr}>"
+    if plan.queue_kind == 2:
+        qr = 8 + plan.queue_regs if plan.queue_regs else (-2 if plan.visited_global else -1)
+        kind = "union W in registers" if plan.queue_regs else "union W in tiers"
+    else:
+        qr = plan.queue_regs
+        kind = "q, topk in registers" if qr else "q, topk in tiers"
+    return f"song_search_kernel<NCH={plan.row_chunks},{met},{visited.upper()},QR={qr}> ({kind})"
 
 
 # ------------------------------------------------------- dataset sharding
@@ -631,6 +636,7 @@ def run_song(args, ws, rank, local, log):
             f"recall_at_{K}": round(rec, 4), "recall_sweep": sweep, "visited": args.visited,
             "visited_cap": args.visited_cap or "default (lazy deletion, reading R14)",
             "visited_cap_resolved": cap, "queue_kind": ["registers", "separate q, topk", "bounded union (R17)"][qkind],
+            "queue_regs": int(plan_op.queue_regs),
             "l2": "flushed between timed steps (512 MiB write)",
             "parallelism": f"query-sharded dp{ws} (graph replicated per GPU)",
         },
@@ -644,7 +650,7 @@ def run_song(args, ws, rank, local, log):
                               f"frac counts the {nq // reps} unique queries' bytes; the {reps} "
                               f"replicas of each re-read its rows from L2")} if reps > 1 else {}),
             "traffic": traffic,
-            "kernel": kernel_name(cfg, L_op, args.visited), "peak_source": peak_src,
+            "kernel": kernel_name(cfg, plan_op, args.visited), "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "n_dist": n_dist, "n_exp": n_exp,
             "kernel_ms": round(kernel_s * 1e3, 4),
             "kernel_ms_note": "whole step on the launching stream: search kernel + outlier-first scheduling kernels (conservative for the search kernel alone)",

@@ -105,11 +105,14 @@ typedef struct song_search_params {
                               float index (else SONG_EUNSUPPORTED) */
   int32_t visited_cap;     /* SONG_VISITED_HASH deletion schedule (§IV-E, DESIGN.md
                               reading R14).  0 = lazy deletion with the default capacity
-                              C = 5S/8 for queue_len <= 128, 3S/4 above, where S =
-                              2^ceil(log2(F (2L + 32))) table slots, F = 8 (L <= 64), 4 (L <= 128) or
-                              4/3 (song_search_plan_get reports the C in effect); > 0 =
-                              lazy with C = visited_cap (2L + 32 <= C <= 3S/4,
-                              else SONG_EINVAL); -1 = eager deletion (every evicted vertex
+                              C: separate q / topk (queue_kind SEPARATE) C = 5S/8 for
+                              queue_len <= 128, 3S/4 above, where S = 2^ceil(log2(F (2L +
+                              32))) table slots, F = 8 (L <= 64; 4 for rows of 129-256
+                              floats), 4 (L <= 128) or 4/3; the union (queue_kind UNION,
+                              the default for visited HASH, steps 1): see queue_kind
+                              (song_search_plan_get reports the C in effect); > 0 =
+                              lazy with C = visited_cap (2L + 32 <= C <= 3S/4, or
+                              L + 32 <= C for the union; else SONG_EINVAL); -1 = eager deletion (every evicted vertex
                               erased at once, the paper's literal schedule).  Lazy: the
                               erasures are applied together (visited := ids(q) ∪
                               ids(topk)) when the selected candidates of an iteration
@@ -128,9 +131,11 @@ typedef struct song_search_params {
                               in 4096 log-spaced key bins.  Codes indexes always use
                               batch order. */
   int32_t queue_kind;      /* how q and topk are held (results never depend on it).
-                              SONG_QUEUE_AUTO (0, default): registers for queue_len <=
-                              128; above, with visited HASH and steps <= 1, the bounded
-                              union, else separate shared-memory q and topk.
+                              SONG_QUEUE_AUTO (0, default): with visited HASH and steps
+                              <= 1 the bounded union (W in 1, 2 or 4 registers per lane
+                              for queue_len <= 128, in shared memory above); otherwise
+                              separate q and topk, in registers for queue_len <= 128,
+                              in shared memory above.
                               SONG_QUEUE_SEPARATE: q and topk as the paper keeps them
                               (§IV-C), each bounded at L.  SONG_QUEUE_UNION (DESIGN.md
                               reading R17): ONE list of the L best keys of q ∪ topk,
@@ -138,7 +143,8 @@ typedef struct song_search_params {
                               unpopped key, the search stops when none is left; the
                               hash then holds <= L + 32 live ids (lazy capacity C in
                               [L + 32, 3S/4], default 3S/4, S = 2^ceil(log2(8 (L + 32)
-                              / 3))) and a vertex dropped from the list is recomputed if
+                              / 3)) above queue_len 128 and the separate queues' S up
+                              to 128) and a vertex dropped from the list is recomputed if
                               met again (counters differ, results do not).  UNION needs
                               visited HASH and steps <= 1 (else SONG_EUNSUPPORTED). */
 } song_search_params;

@@ -40,7 +40,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB
     newest = max(os.path.getmtime(p) for p in DEPS)
     if not force and os.path.exists(out) and os.path.getmtime(out) >= newest:
         return out
-    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.split("=")[0] for d in defines)
+    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
     os.makedirs(build_dir, exist_ok=True)
     with concurrent.futures.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
         results = list(ex.map(lambda src: _compile(src, defines, build_dir), SOURCES))

@@ -74,6 +74,16 @@ int launch_q(song_index* ix, const SearchArgs& a, int qr, int warps, int bps, in
     case 1: return launch_t<NCH, METRIC, VK, 1, MS>(ix, a, warps, bps, sms, st);
     case 2: return launch_t<NCH, METRIC, VK, 2, MS>(ix, a, warps, bps, sms, st);
     case 4: return launch_t<NCH, METRIC, VK, 4, MS>(ix, a, warps, bps, sms, st);
+    case 9:   // reading R17 with W in 1, 2 or 4 registers per lane (queue_len <= 128)
+    case 10:
+    case 12:
+      if constexpr (VK == VK_HASH && !MS) {
+        if (qr == 9) return launch_t<NCH, METRIC, VK, 9, false>(ix, a, warps, bps, sms, st);
+        if (qr == 10) return launch_t<NCH, METRIC, VK, 10, false>(ix, a, warps, bps, sms, st);
+        return launch_t<NCH, METRIC, VK, 12, false>(ix, a, warps, bps, sms, st);
+      } else {
+        return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH, steps 1");
+      }
     case -1:  // reading R17 (one bounded list of q ∪ topk): the hash visited set only
     case -2:  // ... with the visited table in global memory
       if constexpr (VK == VK_HASH && !MS) {

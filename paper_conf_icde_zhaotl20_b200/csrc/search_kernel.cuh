@@ -755,11 +755,19 @@ constexpr bool kDistTeam = false;  // lane-slice distance path (query in registe
 #ifndef SONG_UNION_WIDE_ROWS
 #define SONG_UNION_WIDE_ROWS 4
 #endif
+// rows per round for rows wider than 256 floats (GIST-shaped, 3.75 KB rows):
+// 8 rows in flight per dependent round trip beat 4 rows at twice the resident
+// warps (GIST L = 24: 2.38 M -> 2.67 M QPS; 16 rows: 1.55 M; 2 rows: 2.13 M;
+// profiles/r03n_*, r03o_*)
+#ifndef SONG_XWIDE_ROWS
+#define SONG_XWIDE_ROWS 8
+#endif
 template <int NCH, bool UNION = false>
 struct StageRows {  // rows per round: SONG_STAGE_ROWS for 128-float rows, 4 for wider ones
   // (NYTimes-shaped, 256 floats: 8 -> 4 rows frees 4 KB per warp, 14 -> 19 resident warps,
   // +12 % QPS; SIFT-shaped rows keep 8: at equal residency 4 rows cost 9 %)
-  static constexpr int R = (NCH >= 2) ? (UNION ? SONG_UNION_WIDE_ROWS : 4) : SONG_STAGE_ROWS;
+  static constexpr int R = (NCH >= 2) ? (UNION ? SONG_UNION_WIDE_ROWS : NCH >= 4 ? SONG_XWIDE_ROWS : 4)
+                                      : SONG_STAGE_ROWS;
   static constexpr int NBUF = SONG_STAGE_BUFS;  // rounds in flight
 };
 
@@ -1127,11 +1135,16 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   extern __shared__ __align__(128) unsigned char smem[];
   constexpr int R = StageRows<NCH, (QR < 0)>::R;
   constexpr bool DEL = (VK == VK_HASH || VK == VK_CUCKOO);  // visited deletion (§IV-E)
-  // QR > 0: q / topk in registers; QR == 0: separate q and topk tiers in
-  // shared memory; QR < 0: reading R17, one bounded list W of q ∪ topk
-  constexpr bool UNQ = QR < 0;
+  // QR in 1..4: q / topk in registers; QR == 0: separate q and topk tiers in
+  // shared memory; QR < 0: reading R17, one bounded list W of q ∪ topk in
+  // shared-memory tiers; QR = 8 + r (r = 1, 2, 4): R17's W in r registers per
+  // lane (queue_len <= 128)
+  constexpr bool RUN = QR > 8;    // R17, W in registers
+  constexpr bool UNQ = QR < 0;    // R17, W in shared-memory tiers
+  constexpr bool UNI = UNQ || RUN;  // R17 semantics (either storage)
+  constexpr bool REG = QR > 0 && !RUN;  // separate q / topk in registers
   constexpr bool GVT = QR == -2;  // R17 with the visited table in global memory
-  constexpr int QRr = QR > 0 ? QR : 1;
+  constexpr int QRr = RUN ? QR - 8 : QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int L = a.L;
@@ -1291,8 +1304,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
     tk_r.clear();
     Tier qg{qa, 0, 0}, tg{tk, 0, 0};  // QR <= 0 (qg is W when UNQ)
     int hint = 0;                      // UNQ: index of W's first unpopped key
-    if (QR > 0) {
+    if (REG) {
       if (lane == 0) q.v[0] = ke;
+    } else if (RUN) {
+      if (lane == 0) q.v[0] = (ke & ~0xffffffffull) | ((uint64_t)(uint32_t)a.entry << 1);
     } else {
       if (lane == 0)
         qa[0] = UNQ ? (ke & ~0xffffffffull) | ((uint64_t)(uint32_t)a.entry << 1) : ke;
@@ -1312,6 +1327,16 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
 #endif
     while (qsize > 0) {
       if (UNQ && hint >= qg.size) break;  // R17: no unpopped key left in W
+      int wpos = 0;  // RUN: W's first unpopped key (bit 0 of a W key = popped)
+      if constexpr (RUN) {
+        wpos = -1;
+#pragma unroll
+        for (int r = QRr - 1; r >= 0; --r) {
+          const unsigned m = __ballot_sync(FULL, (q.v[r] & 1ull) == 0);
+          if (m) wpos = r * 32 + __ffs(m) - 1;
+        }
+        if (wpos < 0) break;  // R17: no unpopped key left in W
+      }
       if (iters >= a.max_iters) {
         capped = true;
         break;
@@ -1319,9 +1344,12 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       ++iters;
       // ---- a3: pop / terminate / topk update (Alg. 1 lines 3-8)
       uint64_t now, tmax;
-      if (QR > 0) {
+      if (REG) {
         now = __shfl_sync(FULL, q.v[0], 0);
         tmax = tk_r.get(L - 1);  // KEY_MAX unless topk is full
+      } else if (RUN) {
+        now = q.get(wpos);  // W's smallest unpopped key (R17 step 2)
+        tmax = KEY_MAX;
       } else if (UNQ) {
         now = qg.at(hint);  // W's smallest unpopped key (R17 step 2)
         tmax = KEY_MAX;
@@ -1336,7 +1364,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       // inserting one vertex multiple times"; the oracle's set semantics)
       bool in_topk = false;
       if constexpr (VK == VK_CUCKOO) {
-        if (QR > 0) {
+        if (REG) {
 #pragma unroll
           for (int r = 0; r < QRr; ++r) in_topk |= __any_sync(FULL, tk_r.v[r] == now);
         } else {
@@ -1345,9 +1373,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
           in_topk = r < tsize && at_r == now;
         }
       }
-      if (QR > 0) {
+      if (REG) {
         if (!in_topk) evicted = tk_r.insert_one(now, L, lane);
         q.pop_front(lane);
+      } else if (RUN) {  // now moves from "q" to "topk" inside W
+#pragma unroll
+        for (int r = 0; r < QRr; ++r)
+          if ((wpos >> 5) == r && lane == (wpos & 31)) q.v[r] |= 1ull;
       } else if (UNQ) {
         qg.set_flag(hint, lane);  // now moves from "q" to "topk" inside W
         hint = qg.next_unpopped(hint + 1, lane);
@@ -1361,14 +1393,14 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       // multi-step probing (§V, R13): up to a.steps pops, each checked
       // against the termination rule with topk as the previous pops left it
       int npop = 1;
-      int popid = UNQ ? wkey_id(now) : key_id(now);  // lane i < npop: id of the i-th popped vertex
+      int popid = UNI ? wkey_id(now) : key_id(now);  // lane i < npop: id of the i-th popped vertex
       if constexpr (MS) {
         for (; npop < a.steps && npop < qsize; ++npop) {
-          const uint64_t nx = (QR > 0) ? __shfl_sync(FULL, q.v[0], 0) : qg.at(0);
-          const uint64_t tm = (QR > 0) ? tk_r.get(L - 1) : ((tsize == L) ? tg.at(L - 1) : KEY_MAX);
+          const uint64_t nx = REG ? __shfl_sync(FULL, q.v[0], 0) : qg.at(0);
+          const uint64_t tm = REG ? tk_r.get(L - 1) : ((tsize == L) ? tg.at(L - 1) : KEY_MAX);
           if (tm < nx) break;
           uint64_t ev1;
-          if (QR > 0) {
+          if (REG) {
             ev1 = tk_r.insert_one(nx, L, lane);
             q.pop_front(lane);
           } else {
@@ -1446,12 +1478,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       SONG_ST_MARK(2);
       // ---- a6: maintenance (§IV-C/D/E)
       const int myid = lane < nc ? cidg[lane] : -1;
-      uint64_t key = lane < nc ? (UNQ ? make_wkey(dist, myid) : make_key(dist, myid)) : KEY_MAX;
+      uint64_t key = lane < nc ? (UNI ? make_wkey(dist, myid) : make_key(dist, myid)) : KEY_MAX;
       // selected insertion threshold: topk's max once topk is full;
       // R17: W's max once W is full
-      const uint64_t thr = UNQ ? ((a.sel && qg.size == L) ? qg.at(L - 1) : KEY_MAX)
-                               : (a.sel && tsize == L)
-                                     ? (QR > 0 ? tk_r.get(L - 1) : tg.at(L - 1))
+      const uint64_t thr = RUN   ? ((a.sel && qsize == L) ? q.get(L - 1) : KEY_MAX)
+                           : UNQ ? ((a.sel && qg.size == L) ? qg.at(L - 1) : KEY_MAX)
+                                 : (a.sel && tsize == L)
+                                     ? (REG ? tk_r.get(L - 1) : tg.at(L - 1))
                                      : KEY_MAX;
       // selected insertion: filtered only when worse than ALL of topk
       // (a key equal to topk's max can only arise from a filter false negative)
@@ -1461,12 +1494,21 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if (!sel) key = KEY_MAX;
       // prefetch the adjacency row of the next head = min(q head, best new key)
       if (last_group) {
-        uint64_t qhead = (QR > 0)  ? __shfl_sync(FULL, q.v[0], 0)
-                         : UNQ     ? (hint < qg.size ? qg.at(hint) : KEY_MAX)
-                         : (na_g > 0 ? qg.at(0) : KEY_MAX);
+        uint64_t qhead = REG   ? __shfl_sync(FULL, q.v[0], 0)
+                         : UNQ ? (hint < qg.size ? qg.at(hint) : KEY_MAX)
+                               : (na_g > 0 ? qg.at(0) : KEY_MAX);
+        if constexpr (RUN) {  // W's first unpopped key after this pop
+          qhead = KEY_MAX;
+#pragma unroll
+          for (int r = QRr - 1; r >= 0; --r) {
+            const unsigned m = __ballot_sync(FULL, (q.v[r] & 1ull) == 0);
+            const uint64_t h = __shfl_sync(FULL, q.v[r], m ? __ffs(m) - 1 : 0);
+            if (m) qhead = h;
+          }
+        }
         uint64_t nxt = umin64(qhead, warp_min_key(key));
         if (nxt != KEY_MAX && lane < a.degree)
-          adjv = __ldg(a.adj + (int64_t)(UNQ ? wkey_id(nxt) : key_id(nxt)) * a.degree + lane);
+          adjv = __ldg(a.adj + (int64_t)(UNI ? wkey_id(nxt) : key_id(nxt)) * a.degree + lane);
         else
           adjv = -1;
       }
@@ -1489,8 +1531,8 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
         if constexpr (VK == VK_HASH) {
           // R17 lazy: every candidate is marked visited (a skipped key can
           // never enter W again), so the capacity check counts all of them
-          const bool ins = (UNQ && a.lazy) ? lane < nc : sel;
-          const int nins = (UNQ && a.lazy) ? nc : ns;
+          const bool ins = (UNI && a.lazy) ? lane < nc : sel;
+          const int nins = (UNI && a.lazy) ? nc : ns;
           bool rebuilt = false;
           if (used + nins > a.rebuild_at) {
             rebuilt = true;
@@ -1498,12 +1540,15 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             // (lazy deletion, R14): rebuild visited = ids(q) ∪ ids(topk)
             hs.clear(lane);
             __syncwarp();
-            if (QR > 0) {
+            if (REG) {
 #pragma unroll
               for (int r = 0; r < QRr; ++r) {
                 hs.insert(key_id(q.v[r]), q.v[r] != KEY_MAX);
                 hs.insert(key_id(tk_r.v[r]), tk_r.v[r] != KEY_MAX);
               }
+            } else if (RUN) {  // R17: visited := ids(W)
+#pragma unroll
+              for (int r = 0; r < QRr; ++r) hs.insert(wkey_id(q.v[r]), q.v[r] != KEY_MAX);
             } else if (UNQ) {  // R17: visited := ids(W)
               for (int i0 = 0; i0 < qg.size; i0 += 32) {
                 const uint64_t kw = qg.at(i0 + lane < qg.size ? i0 + lane : 0);  // (all lanes)
@@ -1519,7 +1564,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
                 hs.insert(key_id(kt), i0 + lane < tsize);
               }
             }
-            used = UNQ ? qg.size : na_g + tsize;
+            used = RUN ? qsize : UNQ ? qg.size : na_g + tsize;
             __syncwarp();
           }
           if (GVT && a.lazy && !rebuilt) {
@@ -1540,7 +1585,27 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
         }
       };
       int qsize_new = min(na_g + ns, L);
-      if (QR > 0) {
+      if (RUN) {  // R17, W in registers: merge the selected keys, drop beyond L
+        visit_selected();  // (lazy: every candidate is marked visited)
+        qsize_new = min(qsize + ns, L);
+        if (ns > 0) {
+          if (sel) keys32[__popc(smask & lt)] = key;
+          __syncwarp();
+          uint64_t k2 = lane < ns ? keys32[lane] : KEY_MAX;
+          __syncwarp();
+          k2 = sort_prefix(k2, ns, lane);
+          const uint64_t sdesc = __shfl_sync(FULL, k2, 31 - lane);  // descending
+          uint64_t out;
+          merge_into<QRr>(q, sdesc, lane, out);
+#pragma unroll
+          for (int r = 0; r < QRr; ++r) {
+            const bool beyond = r * 32 + lane >= L && q.v[r] != KEY_MAX;
+            if constexpr (VK == VK_HASH) hs.erase(wkey_id(q.v[r]), beyond && !a.lazy);  // [del]
+            q.v[r] = r * 32 + lane >= L ? KEY_MAX : q.v[r];
+          }
+          if constexpr (VK == VK_HASH) hs.erase(wkey_id(out), out != KEY_MAX && !a.lazy);
+        }
+      } else if (REG) {
         if (ns > 0) {  // (ns == 0: q only lost its head, nothing to insert/evict)
           visit_selected();
           // Cuckoo false negatives: a selected key may already be in q
@@ -1699,7 +1764,25 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       for (int k = 0; k < 4; ++k) atomicAdd(a.stage_cycles + k, st_acc[k]);
 #endif
     // ---- a7: output the first K of topk (Alg. 1 line 17)
-    if (QR > 0) {
+    if (RUN) {  // R17: the first K popped keys of W (all of W at a normal stop)
+      int outn = 0;
+#pragma unroll
+      for (int r = 0; r < QRr; ++r) {
+        const uint64_t k = q.v[r];
+        const bool pp = k != KEY_MAX && (k & 1ull);
+        const unsigned m = __ballot_sync(FULL, pp);
+        const int o = outn + __popc(m & lt);
+        if (pp && o < a.K) {
+          ids_o[o] = wkey_id(k) + a.id_offset;
+          dists_o[o] = ord2f((uint32_t)(k >> 32));
+        }
+        outn += __popc(m);
+      }
+      for (int i = min(outn, a.K) + lane; i < a.K; i += 32) {
+        ids_o[i] = -1;
+        dists_o[i] = __int_as_float(0x7f800000);
+      }
+    } else if (REG) {
 #pragma unroll
       for (int r = 0; r < QRr; ++r) {
         const int i = r * 32 + lane;

@@ -226,18 +226,38 @@ struct Shape {
 #ifndef SONG_HASH_FACTOR_WIDEROW
 #define SONG_HASH_FACTOR_WIDEROW 4
 #endif
+// queue_kind AUTO picks the union with W in registers for queue_len in
+// [SONG_RUN_AUTO_MIN_L, 128] (above 128 the union is the default anyway).
+// Measured against separate register q / topk at equal table sizes
+// (profiles/r03q_*): SIFT1M L 16 19.6 -> 20.0 M QPS, K = 100 at L 100
+// 5.49 -> 6.00 M, NYTimes L 56 6.39 -> 6.42 M: the pop no longer shifts q
+// and no topk insertion runs (W keeps popped keys in place, flagged)
+#ifndef SONG_RUN_AUTO_MIN_L
+#define SONG_RUN_AUTO_MIN_L 1
+#endif
+// rows wider than 256 floats (GIST-shaped, 8 chunks per lane) keep F = 8: their
+// 8-row stage (30 KB per warp) sets residency anyway, and a smaller table only
+// adds recomputation (GIST L = 24: 2.67 M (F 4) -> 2.86 M QPS, profiles/r03p_*)
+#ifndef SONG_HASH_FACTOR_XWIDE
+#define SONG_HASH_FACTOR_XWIDE 8
+#endif
 int nch_of(int dpad, bool hamming) {
   int n = hamming ? (dpad + 3) / 4 : (dpad + 127) / 128;
   return n <= 1 ? 1 : n <= 2 ? 2 : n <= 4 ? 4 : 8;
 }
 
 int hash_log2_slots(int L, bool uni = false, int nch = 1) {
-  if (uni)
+  // (queue_len <= 128: the union with W in registers takes the table of the
+  // separate register queues — live ids <= L + 32 there, so the load halves
+  // and lazy deletion rebuilds less often; 4x / 8/3x as many slots measured
+  // slower: more shared memory or more recomputation, profiles/r03q_*)
+  if (uni && L > 128)
     return next_pow2_log2((SONG_HASH_UNION_NUM * (L + 32ll) + SONG_HASH_UNION_DEN - 1) /
                           SONG_HASH_UNION_DEN);
   const long long live = 2ll * L + 32;
   if (L > 128) return next_pow2_log2((SONG_HASH_BIG_NUM * live + SONG_HASH_BIG_DEN - 1) / SONG_HASH_BIG_DEN);
   const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE
+                     : nch >= 4 ? SONG_HASH_FACTOR_XWIDE
                      : nch >= 2 ? SONG_HASH_FACTOR_WIDEROW : SONG_HASH_FACTOR;
   return next_pow2_log2(F * live);
 }
@@ -248,6 +268,8 @@ enum QueueKind { QK_REGS = 0, QK_SEPARATE = 1, QK_UNION = 2 };
 int queue_kind_of(int L, int vk, const song_search_params* p) {
   const bool union_ok = vk == song::VK_HASH && p->steps <= 1;
   if (p->queue_kind == SONG_QUEUE_UNION && union_ok) return QK_UNION;
+  if (L <= 128 && L >= SONG_RUN_AUTO_MIN_L && p->queue_kind == SONG_QUEUE_AUTO && union_ok)
+    return QK_UNION;
   if (L <= 128) return QK_REGS;
   if (p->queue_kind == SONG_QUEUE_AUTO && union_ok) return QK_UNION;
   return QK_SEPARATE;
@@ -296,11 +318,15 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   s.nch = nch_of(dpad, hamming);
   const int qk = queue_kind_of(L, vk, p);
   s.qk = qk;
-  s.qr = qk == QK_UNION ? -1 : qk == QK_SEPARATE ? 0 : L <= 32 ? 1 : L <= 64 ? 2 : 4;
+  const int regs = L <= 32 ? 1 : L <= 64 ? 2 : 4;
+  // QR codes of the kernel: 1/2/4 registers, 0 tiers, -1 union in tiers,
+  // 8 + regs the union with W in registers (queue_len <= 128)
+  s.qr = qk == QK_UNION ? (L <= 128 ? 8 + regs : -1) : qk == QK_SEPARATE ? 0 : regs;
 #ifndef SONG_UNION_WIDE_ROWS
 #define SONG_UNION_WIDE_ROWS 4
 #endif
-  const int rows = s.nch >= 2 ? (s.qr < 0 ? SONG_UNION_WIDE_ROWS : 4) : SONG_STAGE_ROWS;  // StageRows<NCH, UNION>::R
+  const int rows = s.nch >= 2 ? (s.qr < 0 ? SONG_UNION_WIDE_ROWS : s.nch >= 4 ? SONG_XWIDE_ROWS : 4)
+                              : SONG_STAGE_ROWS;  // StageRows<NCH, UNION>::R
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
@@ -851,7 +877,7 @@ int song_search_plan_get(const song_search_params* p, int32_t dim, int32_t metri
   const int vk = vk_of(p);
   out->visited_log2 = sh.table_log2;
   out->visited_cap = vk != song::VK_HASH ? 0 : sh.lazy ? sh.rebuild_at : -1;
-  out->queue_regs = sh.qr > 0 ? sh.qr : 0;
+  out->queue_regs = sh.qr > 8 ? sh.qr - 8 : sh.qr > 0 ? sh.qr : 0;
   out->queue_kind = sh.qk;
   out->visited_global = sh.gvis;
   out->row_chunks = sh.nch;

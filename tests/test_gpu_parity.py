@@ -120,12 +120,24 @@ def test_fig1_toy_on_gpu(visited):
                       **oracle_kw(visited, 3, idx=idx))
     assert_exact((ids, d, c), o)
     if visited == "hash":
-        # the paper's literal (eager) deletion: Fig. 4(c), 12 distances, 4 expansions
-        ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited, visited_cap=-1)
+        # the paper's literal structures (separate q and topk) with its literal
+        # (eager) deletion: Fig. 4(c), 12 distances, 4 expansions
+        ids, d, c = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited, visited_cap=-1,
+                               queue_kind="separate")
         assert [int(x) + 1 for x in ids[0]] == result
         assert c[0].tolist() == [12, 4]
         # lazy deletion with the default capacity (R14): no vertex recomputed here
-        assert gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3)[2][0].tolist() == [10, 4]
+        assert gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3,
+                          queue_kind="separate")[2][0].tolist() == [10, 4]
+        # the bounded union (R17, the default): the same ids and pops; its eager
+        # deletion differs from Fig. 4(c)'s (a key leaves W, not q or topk)
+        for cap in (0, -1):
+            g = gpu_search(idx, np.zeros((1, 1), np.float32), 3, 3, visited, visited_cap=cap,
+                           queue_kind="union")
+            assert [int(x) + 1 for x in g[0][0]] == result and g[2][0][1] == 4
+            o = oracle.search(data, adj, np.zeros((1, 1), np.float32), 3, 3,
+                              **oracle_kw(visited, 3, visited_cap=cap, queue_kind="union", idx=idx))
+            assert_exact(g, o)
 
 
 # ----------------------------------------------------------------- tiny config
@@ -351,6 +363,31 @@ def test_union_queue_bit_exact(sift100k, L, cap):
     assert o is not None and s.plan(s.Params(K=1, queue_len=L), 128).queue_kind == 2
     assert_exact(g, o)
     sep = gpu_search(idx, qn, cfg.K, L, "hash", queue_kind="separate")
+    np.testing.assert_array_equal(g[0], sep[0])
+    np.testing.assert_array_equal(g[1], sep[1])
+    np.testing.assert_array_equal(g[2][:, 1], sep[2][:, 1])  # the same popped sequence
+
+
+@pytest.mark.parametrize("L", [10, 16, 48, 100, 128])
+@pytest.mark.parametrize("cap", [0, -1, "min"])
+def test_register_union_bit_exact(sift100k, L, cap):
+    """Reading R17 with W in registers (queue_kind "union" at queue_len <=
+    128): bit-exact against the oracle's bounded-union mode, every deletion
+    schedule, and the same results and pops as the separate register q /
+    topk of §IV-C."""
+    cfg, x, q, adj = sift100k
+    cap = L + 32 if cap == "min" else cap
+    s = song()
+    idx = s.SongIndex(x, adj)
+    K = min(cfg.K, L)
+    xn, an, qn = x.cpu().numpy(), adj.cpu().numpy(), q.cpu().numpy()
+    pl = idx.plan(s.Params(K=K, queue_len=L, queue_kind="union"))
+    assert pl.queue_kind == 2 and pl.queue_regs == (1 if L <= 32 else 2 if L <= 64 else 4)
+    g = gpu_search(idx, qn, K, L, "hash", visited_cap=cap, queue_kind="union")
+    o = oracle.search(xn, an, qn, K, L, nthreads=8,
+                      **oracle_kw("hash", L, visited_cap=cap, queue_kind="union", idx=idx))
+    assert_exact(g, o)
+    sep = gpu_search(idx, qn, K, L, "hash", queue_kind="separate")
     np.testing.assert_array_equal(g[0], sep[0])
     np.testing.assert_array_equal(g[1], sep[1])
     np.testing.assert_array_equal(g[2][:, 1], sep[2][:, 1])  # the same popped sequence

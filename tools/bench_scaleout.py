@@ -213,11 +213,11 @@ def main():
                 import oracle
                 pick = np.arange(0, a.nq, max(1, a.nq // a.parity_sample))[:a.parity_sample]
                 gi, gd, gc = (t.cpu().numpy() for t in idx.search(q, params=p, counters=True))
-                cap = int(__import__("paper_conf_icde_zhaotl20_b200.song", fromlist=["x"]).default_visited_cap(L_op, cfg.dim, cfg.metric))
                 t1 = time.time()
                 oi, od, oc, _ = oracle.search(x.cpu().numpy(), adj_host, q.cpu().numpy()[pick], 10,
-                                              L_op, flags=oracle.OPTIMIZED_LAZY, lazy_cap=cap,
-                                              nthreads=os.cpu_count() or 8)
+                                              L_op, nthreads=os.cpu_count() or 8,
+                                              **bench.oracle_mode(L_op, int(idx.plan(p).visited_cap),
+                                                                  queue_kind=int(idx.plan(p).queue_kind)))
                 row["parity_sample"] = {
                     "queries": len(pick), "oracle_s": round(time.time() - t1, 1),
                     "ids_equal": float((gi[pick] == oi).all(1).mean()),
