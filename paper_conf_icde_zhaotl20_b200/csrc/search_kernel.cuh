@@ -1123,9 +1123,17 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 // shared-memory queues (QR == 0) are held to <= 20 warps per SM by their
 // shared memory anyway: 5 CTAs give them 102 registers (the ring moves keep
 // 4 keys per lane in flight) instead of spilling at 80
+// the union with W in registers (QR > 8) needs fewer registers than separate
+// q / topk: 7 CTAs (72 registers, 28 warps per SM where shared memory allows)
+// measured SIFT1M L 16 20.0 -> 20.6 M QPS (8 CTAs / 64 registers: 20.4 M;
+// K = 100 and NYTimes, held by shared memory, unchanged; profiles/r03s_*)
+#ifndef SONG_RUN_LB_BLOCKS
+#define SONG_RUN_LB_BLOCKS 7
+#endif
 template <int NCH, int QR = 1>
 struct MinBlocks {
-  static constexpr int value = NCH >= 4 ? 4 : (QR == 0 ? 5 : SONG_LB_BLOCKS);
+  static constexpr int value =
+      NCH >= 4 ? 4 : (QR == 0 ? 5 : QR > 8 ? SONG_RUN_LB_BLOCKS : SONG_LB_BLOCKS);
 };
 // MS: multi-step probing (a.steps pops per iteration, <= MAX_STEPS; §V)
 constexpr int MAX_STEPS = 4;
