@@ -77,9 +77,13 @@ int launch_q(song_index* ix, const SearchArgs& a, int qr, int warps, int bps, in
     case 9:   // reading R17 with W in 1, 2 or 4 registers per lane (queue_len <= 128)
     case 10:
     case 12:
+    case 16:
       if constexpr (VK == VK_HASH && !MS) {
         if (qr == 9) return launch_t<NCH, METRIC, VK, 9, false>(ix, a, warps, bps, sms, st);
         if (qr == 10) return launch_t<NCH, METRIC, VK, 10, false>(ix, a, warps, bps, sms, st);
+#if SONG_RUN_MAX_L > 128
+        if (qr == 16) return launch_t<NCH, METRIC, VK, 16, false>(ix, a, warps, bps, sms, st);
+#endif
         return launch_t<NCH, METRIC, VK, 12, false>(ix, a, warps, bps, sms, st);
       } else {
         return fail(SONG_EUNSUPPORTED, "the bounded-union queue needs visited HASH, steps 1");

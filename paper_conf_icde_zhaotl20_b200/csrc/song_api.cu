@@ -318,10 +318,10 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   s.nch = nch_of(dpad, hamming);
   const int qk = queue_kind_of(L, vk, p);
   s.qk = qk;
-  const int regs = L <= 32 ? 1 : L <= 64 ? 2 : 4;
+  const int regs = L <= 32 ? 1 : L <= 64 ? 2 : L <= 128 ? 4 : 8;
   // QR codes of the kernel: 1/2/4 registers, 0 tiers, -1 union in tiers,
   // 8 + regs the union with W in registers (queue_len <= 128)
-  s.qr = qk == QK_UNION ? (L <= 128 ? 8 + regs : -1) : qk == QK_SEPARATE ? 0 : regs;
+  s.qr = qk == QK_UNION ? (L <= SONG_RUN_MAX_L ? 8 + regs : -1) : qk == QK_SEPARATE ? 0 : regs;
 #ifndef SONG_UNION_WIDE_ROWS
 #define SONG_UNION_WIDE_ROWS 4
 #endif

@@ -56,6 +56,12 @@ struct song_index {
   cudaEvent_t ev_h2d = nullptr, ev_done = nullptr, ev_out = nullptr;
 };
 
+// the bounded union (reading R17) keeps W in registers up to this queue_len
+// (128: 4 u64 per lane; 256: 8), in shared-memory tiers above
+#ifndef SONG_RUN_MAX_L
+#define SONG_RUN_MAX_L 128
+#endif
+
 namespace song {
 int fail(int code, const char* fmt, ...);
 // non-owning search index over device rows (the batched graph builder, R16):
