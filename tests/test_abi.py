@@ -53,6 +53,26 @@ def test_argument_errors_need_no_gpu():
     p = song.SearchParams()
     lib.song_default_params(ctypes.byref(p), 10, 64)
     assert (p.K, p.queue_len, p.visited, p.entry, p.id_offset, p.steps) == (10, 64, 0, 0, 0, 0)
+    buf = (ctypes.c_float * 8)()
+    rc = lib.song_search_pipelined(None, ctypes.byref(p), buf, 1, 1, buf, buf)
+    assert rc == -1 and b"NULL" in lib.song_last_error()
+
+
+def test_union_is_the_default_queue():
+    """Reading R17 (one bounded list W of q and topk) is what the library runs
+    by default with the hash visited set and one pop per iteration: in
+    registers up to queue_len 128, in shared-memory tiers above; the paper's
+    separate q / topk on request, and for the other visited kinds."""
+    from paper_conf_icde_zhaotl20_b200 import song
+    for L, regs in ((16, 1), (33, 2), (100, 4), (128, 4), (160, 0), (1280, 0)):
+        pl = song.plan(song.Params(K=10, queue_len=L), 128)
+        assert (pl.queue_kind, pl.queue_regs) == (2, regs), L
+    sep = song.plan(song.Params(K=10, queue_len=64, queue_kind="separate"), 128)
+    assert (sep.queue_kind, sep.queue_regs) == (0, 2)
+    bl = song.plan(song.Params(K=10, queue_len=64, visited="bloom"), 128)
+    assert bl.queue_kind == 0
+    ms = song.plan(song.Params(K=10, queue_len=64, steps=2), 128)
+    assert ms.queue_kind == 0
 
 
 def test_params_struct_layout_matches_header(tmp_path):
