@@ -103,6 +103,8 @@ def parse():
     ap.add_argument("--queue-kind", default="auto", choices=["auto", "separate", "union"],
                     help="song_search_params.queue_kind (results never depend on it)")
     ap.add_argument("--warps-per-block", type=int, default=0)
+    ap.add_argument("--queries-per-warp", type=int, default=0,
+                    help="Fig. 8 packing kernel: 1, 2 or 4 queries per warp (needs --visited-cap -1)")
     ap.add_argument("--blocks-per-sm", type=int, default=0)
     ap.add_argument("--visited-cap", type=int, default=0,
                     help="hash deletion schedule: 0 lazy (default capacity), >0 lazy capacity, "
@@ -480,7 +482,7 @@ def run_song(args, ws, rank, local, log):
         return song.Params(K=cfg.K, queue_len=L, visited=args.visited,
                            warps_per_block=args.warps_per_block, blocks_per_sm=args.blocks_per_sm,
                            visited_cap=args.visited_cap, queue_kind=args.queue_kind,
-                           schedule=args.schedule)
+                           schedule=args.schedule, queries_per_warp=args.queries_per_warp)
 
     # ---- operating point: smallest grid queue_len with recall@10 >= target
     sweep = []
@@ -650,7 +652,10 @@ def run_song(args, ws, rank, local, log):
                               f"frac counts the {nq // reps} unique queries' bytes; the {reps} "
                               f"replicas of each re-read its rows from L2")} if reps > 1 else {}),
             "traffic": traffic,
-            "kernel": kernel_name(cfg, plan_op, args.visited), "peak_source": peak_src,
+            "kernel": (f"song_search_mq_kernel<G={args.queries_per_warp},"
+                       f"{'L2' if cfg.metric == 'l2' else 'DOT'}> (Fig. 8 packing)"
+                       if args.queries_per_warp else kernel_name(cfg, plan_op, args.visited)),
+            "peak_source": peak_src,
             "alg_bytes_per_launch": alg_bytes, "n_dist": n_dist, "n_exp": n_exp,
             "kernel_ms": round(kernel_s * 1e3, 4),
             "kernel_ms_note": "whole step on the launching stream: search kernel + outlier-first scheduling kernels (conservative for the search kernel alone)",
@@ -677,7 +682,8 @@ def run_song(args, ws, rank, local, log):
         # per step: the search kernel, plus the two outlier-first scheduling
         # kernels (order keys + scatter) when the batch outnumbers the resident
         # warps (song.h SONG_SCHEDULE_AUTO)
-        "gpu_launches": args.steps * (3 if nq > 24 * torch.cuda.get_device_properties(dev).multi_processor_count else 1),
+        "gpu_launches": args.steps * (3 if nq > 24 * torch.cuda.get_device_properties(dev).multi_processor_count
+                                      and not args.queries_per_warp else 1),
     }
 
     # ---- the operating point on SURVEY §8(d)'s coarser grid, when it differs

@@ -147,6 +147,18 @@ typedef struct song_search_params {
                               to 128) and a vertex dropped from the list is recomputed if
                               met again (counters differ, results do not).  UNION needs
                               visited HASH and steps <= 1 (else SONG_EUNSUPPORTED). */
+  int32_t queries_per_warp; /* Fig. 8's multi-query packing (§V).
+                              0 (default) = the production kernel (one query per warp,
+                              every stage warp-cooperative).  1, 2 or 4 = the packing
+                              kernel: that many queries per warp, each searched by its
+                              own team of 32 / queries_per_warp lanes with team-scoped
+                              collectives and its own shared-memory q, topk (sorted
+                              arrays) and exact hash; the paper's literal schedule
+                              (separate q / topk, selected insertion, eager deletion).
+                              Needs visited HASH, visited_cap -1, steps <= 1,
+                              queue_kind AUTO or SEPARATE, queue_len <= 128 and a float
+                              index (else SONG_EUNSUPPORTED); results equal the other
+                              kernels', counters equal the eager schedule's. */
 } song_search_params;
 
 #define SONG_QUEUE_AUTO 0

@@ -17,6 +17,7 @@
 #include "rp_kernel.cuh"
 #include "schedule.cuh"
 #include "search_kernel.cuh"
+#include "mq_kernel.cuh"
 #include "song.h"
 
 #include "song_internal.h"
@@ -278,6 +279,18 @@ int queue_kind_of(int L, int vk, const song_search_params* p) {
 Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool hamming) {
   const int steps = p->steps;
   Shape s;
+  if (p->queries_per_warp > 0) {  // Fig. 8's packing kernel (mq_kernel.cuh)
+    s.table_log2 = hash_log2_slots(L, false, nch_of(dpad, hamming));
+    s.rebuild_at = (1 << s.table_log2) / 4;  // tombstones: rebuild at 1/4 load
+    s.lazy = 0;
+    s.qr = 0;
+    s.qk = QK_SEPARATE;
+    s.gvis = 0;
+    s.nch = nch_of(dpad, hamming);
+    s.warps = 4;
+    s.warp_bytes = p->queries_per_warp * song::mq_layout(L, dpad, s.table_log2).total;
+    return s;
+  }
   int tbytes = 0;
   s.rebuild_at = 0;
   if (vk == song::VK_BLOOM) {
@@ -393,6 +406,15 @@ int check_params_common(const song_search_params* p, int metric) {
 
   if (p->schedule < SONG_SCHEDULE_AUTO || p->schedule > SONG_SCHEDULE_OUTLIER_FIRST)
     return fail(SONG_EINVAL, "unknown schedule %d", p->schedule);
+  if (p->queries_per_warp != 0 && p->queries_per_warp != 1 && p->queries_per_warp != 2 &&
+      p->queries_per_warp != 4)
+    return fail(SONG_EINVAL, "queries_per_warp %d not in {0, 1, 2, 4}", p->queries_per_warp);
+  if (p->queries_per_warp > 0 &&
+      (p->visited != SONG_VISITED_HASH || p->visited_cap != -1 || p->steps > 1 ||
+       p->queue_kind == SONG_QUEUE_UNION || p->queue_len > 128 || metric == SONG_HAMMING))
+    return fail(SONG_EUNSUPPORTED,
+                "queries_per_warp > 0 needs visited HASH, visited_cap -1, steps <= 1, queue_kind "
+                "AUTO or SEPARATE, queue_len <= 128 and a float index");
   if (p->steps > SONG_MAX_STEPS)
     return fail(SONG_EUNSUPPORTED, "steps %d > %d", p->steps, SONG_MAX_STEPS);
   if (p->steps > 1 && ((p->visited != SONG_VISITED_HASH && p->visited != SONG_VISITED_BLOOM) ||
@@ -487,6 +509,64 @@ int prepare_order(song_index* ix, const float* q, int64_t nq, cudaStream_t st) {
   return SONG_OK;
 }
 
+// Fig. 8's packing kernel: G = queries_per_warp queries per warp (mq_kernel.cuh)
+template <int G, int METRIC>
+int launch_mq_t(song_index* ix, const song::MqArgs& m, cudaStream_t st) {
+  auto kern = song::song_search_mq_kernel<G, METRIC>;
+  const size_t smem = (size_t)m.team_smem_bytes * G * 4;  // 4 warps per CTA
+  if (smem > 227 * 1024) return fail(SONG_EUNSUPPORTED, "packing kernel needs %zu B per CTA", smem);
+  CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int fit = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&fit, kern, 128, smem));
+  if (fit < 1) return fail(SONG_EUNSUPPORTED, "packing kernel does not fit an SM");
+  const int64_t want = (m.nq + 4 * G - 1) / (4 * G);
+  const int64_t grid = std::min<int64_t>((int64_t)fit * ix->num_sms, want);
+  CUDA_TRY(cudaMemsetAsync(m.ticket, 0, sizeof(unsigned), st));
+  kern<<<(unsigned)grid, 128, smem, st>>>(m);
+  CUDA_TRY(cudaGetLastError());
+  return SONG_OK;
+}
+
+int enqueue_mq(song_index* ix, const song_search_params* p, const Shape& sh,
+               const song::SearchArgs& a, cudaStream_t st) {
+  song::MqArgs m;
+  m.data = a.data;
+  m.adj = a.adj;
+  m.queries = a.queries;
+  m.ids_out = a.ids_out;
+  m.dists_out = a.dists_out;
+  m.counters_out = a.counters_out;
+  m.ticket = a.ticket;
+  m.order = nullptr;
+  m.status = a.status;
+  m.nq = a.nq;
+  m.dim = a.dim;
+  m.dpad = a.dpad;
+  m.degree = a.degree;
+  m.K = a.K;
+  m.L = a.L;
+  m.table_log2 = sh.table_log2;
+  m.rebuild_at = sh.rebuild_at;
+  m.entry = p->entry;
+  m.max_iters = p->max_iters > 0 ? p->max_iters : (1 << 30);
+  m.id_offset = p->id_offset;
+  m.cosine = ix->metric == SONG_COSINE;
+  m.dedup = ix->dedup;
+  m.team_smem_bytes = sh.warp_bytes / p->queries_per_warp;
+  int rc = order_after_last(ix, st);
+  if (rc) return rc;
+  const bool l2 = ix->metric == SONG_L2;
+  switch (p->queries_per_warp) {
+    case 1: rc = l2 ? launch_mq_t<1, song::MET_L2>(ix, m, st) : launch_mq_t<1, song::MET_DOT>(ix, m, st); break;
+    case 2: rc = l2 ? launch_mq_t<2, song::MET_L2>(ix, m, st) : launch_mq_t<2, song::MET_DOT>(ix, m, st); break;
+    default: rc = l2 ? launch_mq_t<4, song::MET_L2>(ix, m, st) : launch_mq_t<4, song::MET_DOT>(ix, m, st); break;
+  }
+  if (rc) return rc;
+  if (!ix->last_done) CUDA_TRY(cudaEventCreateWithFlags(&ix->last_done, cudaEventDisableTiming));
+  CUDA_TRY(cudaEventRecord(ix->last_done, st));
+  return SONG_OK;
+}
+
 int enqueue_search(song_index* ix, const song_search_params* p, const float* q, int64_t nq,
                    int32_t* ids, float* dists, int32_t* counters, cudaStream_t st) {
   song::SearchArgs a;
@@ -531,6 +611,7 @@ int enqueue_search(song_index* ix, const song_search_params* p, const float* q, 
   if (ix->metric == SONG_HAMMING && vk != song::VK_HASH && vk != song::VK_BLOOM)
     return fail(SONG_EUNSUPPORTED, "Hamming indexes support the hash and Bloom visited sets");
   Shape sh = search_shape(p->queue_len, vk, p, ix->dpad, ix->metric == SONG_HAMMING);
+  if (p->queries_per_warp > 0) return enqueue_mq(ix, p, sh, a, st);
   a.table_log2 = sh.table_log2;
   a.rebuild_at = sh.rebuild_at;
   a.lazy = sh.lazy;

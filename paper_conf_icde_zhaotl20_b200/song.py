@@ -55,7 +55,8 @@ class SearchParams(ctypes.Structure):
                 ("warps_per_block", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
                 ("id_offset", ctypes.c_int32), ("table_log2", ctypes.c_int32),
                 ("steps", ctypes.c_int32), ("visited_cap", ctypes.c_int32),
-                ("schedule", ctypes.c_int32), ("queue_kind", ctypes.c_int32)]
+                ("schedule", ctypes.c_int32), ("queue_kind", ctypes.c_int32),
+                ("queries_per_warp", ctypes.c_int32)]
 
 
 class IndexInfo(ctypes.Structure):
@@ -166,6 +167,7 @@ class Params:
     visited_cap: int = 0  # hash deletion schedule: 0 lazy (default cap), >0 lazy cap, -1 eager
     schedule: str = "auto"  # ticket order: "auto" | "batch" | "outlier_first"
     queue_kind: str = "auto"  # "auto" | "separate" (q, topk) | "union" (reading R17)
+    queries_per_warp: int = 0  # Fig. 8 packing kernel: 1, 2 or 4 queries per warp (0 = default kernel)
 
     def to_c(self) -> SearchParams:
         p = SearchParams()
@@ -182,6 +184,7 @@ class Params:
         p.visited_cap = self.visited_cap
         p.schedule = SCHEDULES[self.schedule]
         p.queue_kind = QUEUE_KINDS[self.queue_kind]
+        p.queries_per_warp = self.queries_per_warp
         return p
 
 

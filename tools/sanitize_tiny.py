@@ -3,8 +3,9 @@
 
     compute-sanitizer --tool racecheck python tools/sanitize_tiny.py
 
-tiny-config search through every visited kind and queue kind (registers,
-separate shared-memory q / topk, the bounded union), multi-step probing,
+tiny-config search through every visited kind and queue kind (separate
+register or shared-memory q / topk, the bounded union in registers or tiers),
+multi-step probing, the pipelined host-buffer path,
 Hamming codes, the three graph builders, both merges.  Exits non-zero if a
 result disagrees with the oracle on the integer-valued sample."""
 from __future__ import annotations
@@ -41,6 +42,8 @@ def main():
     bad = 0
     cases = [("hash", 24, {}), ("hash", 100, {}), ("hash", 200, {}),
              ("hash", 200, {"queue_kind": "separate"}), ("hash", 40, {"queue_kind": "union"}),
+             ("hash", 24, {"queue_kind": "separate"}), ("hash", 100, {"queue_kind": "separate"}),
+             ("hash", 100, {"visited_cap": -1}),
              ("hash", 64, {"visited_cap": -1}), ("bloom", 48, {}), ("hashtable", 48, {}),
              ("hashtable-sel", 200, {}), ("cuckoo", 48, {}), ("cuckoo", 200, {}),
              ("hash", 48, {"steps": 2})]
@@ -67,6 +70,14 @@ def main():
     ptr = torch.tensor([ids.data_ptr(), ids2.data_ptr()], dtype=torch.int64, device="cuda")
     dptr = torch.tensor([d.data_ptr(), d.data_ptr()], dtype=torch.int64, device="cuda")
     song.merge_topk_peers(ptr, dptr, q.shape[0], 10, 10)
+    # the pipelined host-buffer path: two lanes, copy streams, concurrent grids
+    pp = song.Params(K=10, queue_len=24)
+    qb = np.ascontiguousarray(np.stack([q, q[::-1], q]))
+    pi, pd = idx.search_pipelined(qb, pp)
+    ref = idx.search(qt, params=pp)[0].cpu().numpy()
+    ok = (pi[0] == ref).all() and (pi[1] == ref[::-1]).all() and (pi[2] == ref).all()
+    print("pipelined", "ok" if ok else "MISMATCH", flush=True)
+    bad += not ok
     torch.cuda.synchronize()
     print("sanitize_tiny done,", bad, "mismatches", flush=True)
     sys.exit(1 if bad else 0)
