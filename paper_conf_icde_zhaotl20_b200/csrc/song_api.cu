@@ -1191,6 +1191,79 @@ int ensure_twin(song_index* ix) {
   t->last_stream = t->stream;
   return SONG_OK;
 }
+// host batches streamed through two lanes: chunk b = queries [b * chunk,
+// min(total, (b + 1) * chunk)); its HtoD runs on the copy stream once its
+// lane's previous search has read the lane's query buffer, its search on the
+// lane's compute stream, its DtoH on the other copy stream (song.h,
+// song_search_pipelined).  Params are checked by the caller.
+int run_pipeline(song_index* ix, const song_search_params* p, const float* queries,
+                 int64_t nchunks, int64_t chunk, int64_t total, int32_t* ids_out,
+                 float* dists_out) {
+  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
+  const size_t qrow = (size_t)qdim * sizeof(float), orow = (size_t)p->K * sizeof(int32_t);
+  const int nl = nchunks > 1 ? 2 : 1;
+  int rc;
+  if (nl == 2) {
+    rc = ensure_twin(ix);
+    if (rc) return rc;
+  }
+  song_index* lane[2] = {ix, ix->twin};
+  if (!ix->h2d) CUDA_TRY(cudaStreamCreateWithFlags(&ix->h2d, cudaStreamNonBlocking));
+  if (!ix->d2h) CUDA_TRY(cudaStreamCreateWithFlags(&ix->d2h, cudaStreamNonBlocking));
+  for (int l = 0; l < nl; ++l) {
+    rc = ensure_io(lane[l], chunk * qrow, chunk * orow);
+    if (!rc) rc = make_events(lane[l]);
+    if (rc) return rc;
+    // after every search enqueued earlier on the index (any stream)
+    if (ix->last_done) CUDA_TRY(cudaStreamWaitEvent(lane[l]->stream, ix->last_done, 0));
+    lane[l]->last_stream = lane[l]->stream;
+  }
+  // the copy streams too: a lane's buffers may still be read by an earlier call
+  if (ix->last_done) {
+    CUDA_TRY(cudaStreamWaitEvent(ix->h2d, ix->last_done, 0));
+    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, ix->last_done, 0));
+  }
+  const char* qh = reinterpret_cast<const char*>(queries);
+  char* ih = reinterpret_cast<char*>(ids_out);
+  char* dh = reinterpret_cast<char*>(dists_out);
+  for (int64_t b = 0; b < nchunks; ++b) {
+    song_index* L = lane[b % nl];
+    cudaStream_t st = L->stream;
+    const int64_t q0 = b * chunk, nq = std::min(total, q0 + chunk) - q0;
+    // HtoD of chunk b once the lane's previous search (b - nl) has read d_q
+    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(ix->h2d, L->ev_done, 0));
+    CUDA_TRY(cudaMemcpyAsync(L->d_q, qh + q0 * qrow, nq * qrow, cudaMemcpyHostToDevice, ix->h2d));
+    CUDA_TRY(cudaEventRecord(L->ev_h2d, ix->h2d));
+    CUDA_TRY(cudaStreamWaitEvent(st, L->ev_h2d, 0));
+    // the lane's outputs once the DtoH of chunk b - nl has read them
+    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(st, L->ev_out, 0));
+    const float* dq = L->d_q;
+    if (ix->metric == SONG_HAMMING) {
+      rc = encode_queries(L, L->d_q, nq, st);
+      if (rc) return rc;
+      dq = reinterpret_cast<const float*>(L->d_qcodes);
+    }
+    rc = enqueue_search(L, p, dq, nq, L->d_ids, L->d_dists, nullptr, st);
+    if (rc) return rc;
+    CUDA_TRY(cudaEventRecord(L->ev_done, st));
+    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, L->ev_done, 0));
+    CUDA_TRY(cudaMemcpyAsync(ih + q0 * orow, L->d_ids, nq * orow, cudaMemcpyDeviceToHost, ix->d2h));
+    CUDA_TRY(cudaMemcpyAsync(dh + q0 * orow, L->d_dists, nq * orow, cudaMemcpyDeviceToHost, ix->d2h));
+    CUDA_TRY(cudaEventRecord(L->ev_out, ix->d2h));
+  }
+  // the last DtoH waits for the last search, which follows every earlier one
+  // on its lane; the other lane's last search precedes its own DtoH on d2h
+  CUDA_TRY(cudaStreamSynchronize(ix->d2h));
+  int st_all = 0;
+  for (int l = 0; l < nl; ++l) {
+    int s = 0;
+    CUDA_TRY(cudaMemcpy(&s, lane[l]->d_status, sizeof s, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemset(lane[l]->d_status, 0, sizeof s));
+    st_all |= s;
+  }
+  ix->last_stream = ix->stream;
+  return status_code(st_all);
+}
 }  // namespace
 
 extern "C" {
@@ -1242,69 +1315,7 @@ int song_search_pipelined(song_index* ix, const song_search_params* p, const flo
   if (rc) return rc;
   if (ix->metric == SONG_HAMMING && !ix->d_R)
     return fail(SONG_EINVAL, "this index holds codes without R: use song_search_codes_ex");
-  const int qdim = ix->metric == SONG_HAMMING ? ix->rp_dim : ix->dim;
-  const size_t qbytes = (size_t)nq * qdim * sizeof(float);
-  const size_t obytes = (size_t)nq * p->K * sizeof(int32_t);
-  const int nl = nbatch > 1 ? 2 : 1;
-  if (nl == 2) {
-    rc = ensure_twin(ix);
-    if (rc) return rc;
-  }
-  song_index* lane[2] = {ix, ix->twin};
-  if (!ix->h2d) CUDA_TRY(cudaStreamCreateWithFlags(&ix->h2d, cudaStreamNonBlocking));
-  if (!ix->d2h) CUDA_TRY(cudaStreamCreateWithFlags(&ix->d2h, cudaStreamNonBlocking));
-  for (int l = 0; l < nl; ++l) {
-    rc = ensure_io(lane[l], qbytes, obytes);
-    if (!rc) rc = make_events(lane[l]);
-    if (rc) return rc;
-    // after every search enqueued earlier on the index (any stream)
-    if (ix->last_done) CUDA_TRY(cudaStreamWaitEvent(lane[l]->stream, ix->last_done, 0));
-    lane[l]->last_stream = lane[l]->stream;
-  }
-  // the copy streams too: a lane's buffers may still be read by an earlier call
-  if (ix->last_done) {
-    CUDA_TRY(cudaStreamWaitEvent(ix->h2d, ix->last_done, 0));
-    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, ix->last_done, 0));
-  }
-  const char* qh = reinterpret_cast<const char*>(queries);
-  char* ih = reinterpret_cast<char*>(ids_out);
-  char* dh = reinterpret_cast<char*>(dists_out);
-  for (int64_t b = 0; b < nbatch; ++b) {
-    song_index* L = lane[b % nl];
-    cudaStream_t st = L->stream;
-    // HtoD of batch b once the lane's previous search (b - nl) has read d_q
-    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(ix->h2d, L->ev_done, 0));
-    CUDA_TRY(cudaMemcpyAsync(L->d_q, qh + b * qbytes, qbytes, cudaMemcpyHostToDevice, ix->h2d));
-    CUDA_TRY(cudaEventRecord(L->ev_h2d, ix->h2d));
-    CUDA_TRY(cudaStreamWaitEvent(st, L->ev_h2d, 0));
-    // the lane's outputs once the DtoH of batch b - nl has read them
-    if (b >= nl) CUDA_TRY(cudaStreamWaitEvent(st, L->ev_out, 0));
-    const float* dq = L->d_q;
-    if (ix->metric == SONG_HAMMING) {
-      rc = encode_queries(L, L->d_q, nq, st);
-      if (rc) return rc;
-      dq = reinterpret_cast<const float*>(L->d_qcodes);
-    }
-    rc = enqueue_search(L, p, dq, nq, L->d_ids, L->d_dists, nullptr, st);
-    if (rc) return rc;
-    CUDA_TRY(cudaEventRecord(L->ev_done, st));
-    CUDA_TRY(cudaStreamWaitEvent(ix->d2h, L->ev_done, 0));
-    CUDA_TRY(cudaMemcpyAsync(ih + b * obytes, L->d_ids, obytes, cudaMemcpyDeviceToHost, ix->d2h));
-    CUDA_TRY(cudaMemcpyAsync(dh + b * obytes, L->d_dists, obytes, cudaMemcpyDeviceToHost, ix->d2h));
-    CUDA_TRY(cudaEventRecord(L->ev_out, ix->d2h));
-  }
-  // the last DtoH waits for the last search, which follows every earlier one
-  // on its lane; the other lane's last search precedes its own DtoH on d2h
-  CUDA_TRY(cudaStreamSynchronize(ix->d2h));
-  int st_all = 0;
-  for (int l = 0; l < nl; ++l) {
-    int s = 0;
-    CUDA_TRY(cudaMemcpy(&s, lane[l]->d_status, sizeof s, cudaMemcpyDeviceToHost));
-    CUDA_TRY(cudaMemset(lane[l]->d_status, 0, sizeof s));
-    st_all |= s;
-  }
-  ix->last_stream = ix->stream;
-  return status_code(st_all);
+  return run_pipeline(ix, p, queries, nbatch, nq, nbatch * nq, ids_out, dists_out);
 }
 
 int song_merge_topk(const int32_t* ids_in, const float* dists_in, int32_t G, int64_t nq,

@@ -284,6 +284,21 @@ def test_pipelined_large_batches_overlap(sift100k):
         np.testing.assert_array_equal(dh[b].numpy(), g[1])
 
 
+def test_search_host_large_batch(sift100k):
+    """song_search on a batch of several resident grids' worth (outlier-first
+    order, a ragged tail) and then a small call: the device search's results."""
+    cfg, x, _, adj = sift100k
+    s = song()
+    _, qbig = make_data(cfg, device="cpu", n=1000, nq=12_001)  # ragged last chunk
+    idx = s.SongIndex(x, adj)
+    hi, hd = idx.search_host(qbig.numpy(), cfg.K, 24)
+    g = gpu_search(idx, qbig.numpy(), cfg.K, 24)
+    np.testing.assert_array_equal(hi, g[0])
+    np.testing.assert_array_equal(hd, g[1])
+    hi2, _ = idx.search_host(qbig.numpy()[:100], cfg.K, 24)  # then a small unchunked call
+    np.testing.assert_array_equal(hi2, g[0][:100])
+
+
 def test_pipelined_argument_errors(sift100k):
     cfg, x, q, adj = sift100k
     s = song()
