@@ -158,7 +158,8 @@ typedef struct song_search_params {
                               Needs visited HASH, visited_cap -1, steps <= 1,
                               queue_kind AUTO or SEPARATE, queue_len <= 128 and a float
                               index (else SONG_EUNSUPPORTED); results equal the other
-                              kernels', counters equal the eager schedule's. */
+                              kernels', counters equal the eager schedule's.  It issues
+                              the batch in batch order (schedule is ignored). */
 } song_search_params;
 
 #define SONG_QUEUE_AUTO 0

@@ -1183,12 +1183,17 @@ int ensure_twin(song_index* ix) {
   t->rp_dim = ix->rp_dim;
   t->d_R = ix->d_R;
   t->d_centroid = ix->d_centroid;
-  ix->twin = t;  // freed with the owner from here on
-  CUDA_TRY(cudaMalloc(&t->d_ticket, sizeof(unsigned)));
-  CUDA_TRY(cudaMalloc(&t->d_status, sizeof(int)));
-  CUDA_TRY(cudaMemset(t->d_status, 0, sizeof(int)));
-  CUDA_TRY(cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking));
+  cudaError_t e = cudaMalloc(&t->d_ticket, sizeof(unsigned));
+  if (e == cudaSuccess) e = cudaMalloc(&t->d_status, sizeof(int));
+  if (e == cudaSuccess) e = cudaMemset(t->d_status, 0, sizeof(int));
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {  // no half-made lane is ever attached to the index
+    free_index(t);
+    return fail(e == cudaErrorMemoryAllocation ? SONG_ENOMEM : SONG_ECUDA, "second lane: %s",
+                cudaGetErrorString(e));
+  }
   t->last_stream = t->stream;
+  ix->twin = t;  // freed with the owner from here on
   return SONG_OK;
 }
 // host batches streamed through two lanes: chunk b = queries [b * chunk,
