@@ -164,3 +164,22 @@ def test_plan_errors_need_no_gpu():
         song.plan(song.Params(K=1, queue_len=10, visited="cuckoo"), 4, "hamming")
     with pytest.raises(song.SongError):
         song.plan(song.Params(K=1, queue_len=10), 2048)
+
+
+def _build_c_example(tmp_path):
+    import subprocess
+    from paper_conf_icde_zhaotl20_b200 import song
+    libdir = os.path.dirname(song.LIB_PATH)
+    exe = str(tmp_path / "search_example")
+    cmd = ["gcc", "-O2", "-std=c99", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"),
+           os.path.join(ROOT, "examples", "search_example.c"), "-L", libdir, "-lsong",
+           f"-Wl,-rpath,{libdir}", "-lm", "-o", exe]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    assert res.returncode == 0, res.stderr
+    return exe
+
+
+def test_c_example_builds_against_the_header(tmp_path):
+    """A plain C program (no Python, no torch) compiles against include/song.h
+    and links libsong.so; tests/test_gpu_c_example.py runs it on a GPU."""
+    assert os.path.exists(_build_c_example(tmp_path))
