@@ -1168,8 +1168,10 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   uint64_t* ev = keys32 + 32;                                           // 32 evicted keys
   // QR == 0 only: q and topk as tiered vectors of ceil(L / 64) blocks
   const int tslots = QR <= 0 ? ((L + 63) >> 6) << 6 : 0;
-  int* cslot = reinterpret_cast<int*>(ev + 32);  // GVT: each candidate's insert slot
-  uint64_t* qa = reinterpret_cast<uint64_t*>(cslot + 32);  // q (or W, R17)
+  // (the evicted-key list only for the Cuckoo filter, the insert slots only
+  // for GVT: the other kernels give those bytes to more resident warps)
+  int* cslot = reinterpret_cast<int*>(ev + (VK == VK_CUCKOO ? 32 : 0));  // GVT: each candidate's insert slot
+  uint64_t* qa = reinterpret_cast<uint64_t*>(cslot + (GVT ? 32 : 0));  // q (or W, R17)
   uint64_t* tk = qa + tslots;                   // topk (QR == 0 only)
   const int tkslots = QR == 0 ? tslots : 0;
   int* table = GVT ? a.gvis + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2)

@@ -343,7 +343,10 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
   const int qsm_bytes = (hamming || !song::kDistTeam) ? 0 : 512 * s.nch;  // query in smem
-  s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 + 32 * 8 + 32 * 4 +
+  // stage, query, 16 B, candidate ids, 32 keys, 32 evicted keys (Cuckoo only),
+  // [32 insert slots: the union with global tables, added below], tiers, table
+  s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 +
+                 (vk == song::VK_CUCKOO ? 32 * 8 : 0) +
                  (s.qr <= 0 ? (s.qr == 0 ? 2 : 1) * (((L + 63) / 64) * 64) * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
@@ -353,7 +356,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
     // when that holds >= 1.5x the resident warps per SM (the union kernels
     // use <= 80 registers: at most 24 warps per SM)
     auto resident = [](int wb) { return std::min(24, (int)((227 * 1024) / (wb + 256))); };
-    const int wb0 = ((s.warp_bytes - tbytes) + 127) & ~127;
+    const int wb0 = ((s.warp_bytes - tbytes + 32 * 4) + 127) & ~127;  // + the insert slots
     if (2 * resident(wb0) >= 3 * resident(s.warp_bytes)) {
       s.gvis = 1;
       s.qr = -2;
