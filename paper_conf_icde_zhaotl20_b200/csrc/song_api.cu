@@ -250,11 +250,14 @@ int nch_of(int dpad, bool hamming) {
 int hash_log2_slots(int L, bool uni = false, int nch = 1) {
   // (queue_len <= 128: the union with W in registers takes the table of the
   // separate register queues — live ids <= L + 32 there, so the load halves
-  // and lazy deletion rebuilds less often; 4x / 8/3x as many slots measured
-  // slower: more shared memory or more recomputation, profiles/r03q_*)
+  // and lazy deletion rebuilds less often; F (L + 32) slots with F = 8/3, 3
+  // or 4 measured slower (more recomputation: K = 100 6.01 -> 5.68 M at F 3,
+  // NYTimes 6.42 -> 6.27 M at F 4, SIFT L 16 20.5 -> 19.7 M at F 4;
+  // profiles/r03q_*, r03ad A/B)
   if (uni && L > 128)
     return next_pow2_log2((SONG_HASH_UNION_NUM * (L + 32ll) + SONG_HASH_UNION_DEN - 1) /
                           SONG_HASH_UNION_DEN);
+
   const long long live = 2ll * L + 32;
   if (L > 128) return next_pow2_log2((SONG_HASH_BIG_NUM * live + SONG_HASH_BIG_DEN - 1) / SONG_HASH_BIG_DEN);
   const long long F = L > 64 ? SONG_HASH_FACTOR_WIDE
