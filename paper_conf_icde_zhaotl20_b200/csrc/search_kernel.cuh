@@ -1123,6 +1123,12 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 // shared-memory queues (QR == 0) are held to <= 20 warps per SM by their
 // shared memory anyway: 5 CTAs give them 102 registers (the ring moves keep
 // 4 keys per lane in flight) instead of spilling at 80
+// union in registers: up to this many selected keys are inserted one at a
+// time (measured 0 / 2 / 4: SIFT L 16 20.75 / 21.01 / 20.87 M QPS, K = 100
+// 6.02 / 6.06 / 6.06 M, NYTimes 6.47 / 6.49 / 6.51 M; profiles r03ae A/B)
+#ifndef SONG_RUN_INS_MAX
+#define SONG_RUN_INS_MAX 2
+#endif
 // the union with W in registers (QR > 8) needs fewer registers than separate
 // q / topk: 7 CTAs (72 registers, 28 warps per SM where shared memory allows)
 // measured SIFT1M L 16 20.0 -> 20.6 M QPS (8 CTAs / 64 registers: 20.4 M;
@@ -1598,7 +1604,22 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       if (RUN) {  // R17, W in registers: merge the selected keys, drop beyond L
         visit_selected();  // (lazy: every candidate is marked visited)
         qsize_new = min(qsize + ns, L);
-        if (ns > 0) {
+        if (ns > 0 && ns <= SONG_RUN_INS_MAX) {
+          // few selected keys: rank + shift each into W instead of sorting
+          // them and running the bitonic merge (the same L smallest stay and
+          // the same keys leave: a key that arrives at a full W behind its
+          // maximum leaves at once)
+          int wsz = qsize;
+          for (unsigned m = smask; m; m &= m - 1) {
+            const uint64_t kj = __shfl_sync(FULL, key, __ffs(m) - 1);
+            uint64_t evk = q.insert_one(kj, L, lane);
+            if (wsz < L)
+              ++wsz;
+            else if (evk == KEY_MAX)
+              evk = kj;
+            if constexpr (VK == VK_HASH) hs.erase(wkey_id(evk), lane == 0 && evk != KEY_MAX && !a.lazy);
+          }
+        } else if (ns > 0) {
           if (sel) keys32[__popc(smask & lt)] = key;
           __syncwarp();
           uint64_t k2 = lane < ns ? keys32[lane] : KEY_MAX;
