@@ -1,0 +1,11 @@
+cd $GRAFT_REPO_ROOT
+SONG_LIB=paper_conf_icde_zhaotl20_b200/libsong_pm.so timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu -x -k "union or edges or bit_exact or toy" > gpurun_out/r03ag_gputests_pm.log 2>&1; tail -1 gpurun_out/r03ag_gputests_pm.log
+run() { SONG_LIB=paper_conf_icde_zhaotl20_b200/$1 timeout 600 python bench.py $2 --steps 20 --warmup 5 --no-parity --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$1', '$3', d['value'], d['ms_per_step'], d['roofline']['n_dist'], d['roofline']['frac'])"; }
+run libsong_base.so "--K 100 --queue-len 100 --cache /tmp/ab_k100.pt" warm > /dev/null
+run libsong_base.so "--config nytimes256 --queue-len 56 --cache /tmp/ab_nyt.pt" warm > /dev/null
+for rep in 1 2; do
+  for lib in libsong_base.so libsong_pm.so; do
+    run $lib "--K 100 --queue-len 100 --cache /tmp/ab_k100.pt" K100
+    run $lib "--config nytimes256 --queue-len 56 --cache /tmp/ab_nyt.pt" NYT56
+  done
+done
