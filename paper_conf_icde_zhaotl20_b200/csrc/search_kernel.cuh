@@ -759,17 +759,24 @@ constexpr bool kDistTeam = false;  // lane-slice distance path (query in registe
 #define SONG_UNION_WIDE_ROWS 4
 #endif
 // rows per round for rows wider than 256 floats (GIST-shaped, 3.75 KB rows):
-// 8 rows in flight per dependent round trip beat 4 rows at twice the resident
-// warps (GIST L = 24: 2.38 M -> 2.67 M QPS; 16 rows: 1.55 M; 2 rows: 2.13 M;
-// profiles/r03n_*, r03o_*)
+// with one bulk L2 prefetch per later-round row, 2 rows per round at 16
+// resident warps beat 4 (11 warps) and 8 (6 warps): GIST L = 24 4.12 / 3.93 /
+// 3.27 M QPS (r03ak); with per-line prefetches 8 rows had won (2.67 vs 2.38 /
+// 2.13 M, r03n / r03o)
 #ifndef SONG_XWIDE_ROWS
-#define SONG_XWIDE_ROWS 8
+#define SONG_XWIDE_ROWS 2
+#endif
+#ifndef SONG_XWIDE_LB_BLOCKS  // CTAs of 128 threads per SM the wide-row kernels are compiled for
+#define SONG_XWIDE_LB_BLOCKS 4
+#endif
+#ifndef SONG_WIDE_ROWS  // rows per round for 129-256 floats (NYTimes / GloVe-shaped)
+#define SONG_WIDE_ROWS 4
 #endif
 template <int NCH, bool UNION = false>
 struct StageRows {  // rows per round: SONG_STAGE_ROWS for 128-float rows, 4 for wider ones
   // (NYTimes-shaped, 256 floats: 8 -> 4 rows frees 4 KB per warp, 14 -> 19 resident warps,
   // +12 % QPS; SIFT-shaped rows keep 8: at equal residency 4 rows cost 9 %)
-  static constexpr int R = (NCH >= 2) ? (UNION ? SONG_UNION_WIDE_ROWS : NCH >= 4 ? SONG_XWIDE_ROWS : 4)
+  static constexpr int R = (NCH >= 2) ? (UNION ? SONG_UNION_WIDE_ROWS : NCH >= 4 ? SONG_XWIDE_ROWS : SONG_WIDE_ROWS)
                                       : SONG_STAGE_ROWS;
   static constexpr int NBUF = SONG_STAGE_BUFS;  // rounds in flight
 };
@@ -1147,7 +1154,7 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 template <int NCH, int QR = 1>
 struct MinBlocks {
   static constexpr int value =
-      NCH >= 4 ? 4 : (QR == 0 ? 5 : QR > 8 ? SONG_RUN_LB_BLOCKS : SONG_LB_BLOCKS);
+      NCH >= 4 ? SONG_XWIDE_LB_BLOCKS : (QR == 0 ? 5 : QR > 8 ? SONG_RUN_LB_BLOCKS : SONG_LB_BLOCKS);
 };
 // MS: multi-step probing (a.steps pops per iteration, <= MAX_STEPS; §V)
 constexpr int MAX_STEPS = 4;

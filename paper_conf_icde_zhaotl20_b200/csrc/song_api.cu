@@ -341,7 +341,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
 #ifndef SONG_UNION_WIDE_ROWS
 #define SONG_UNION_WIDE_ROWS 4
 #endif
-  const int rows = s.nch >= 2 ? (s.qr < 0 ? SONG_UNION_WIDE_ROWS : s.nch >= 4 ? SONG_XWIDE_ROWS : 4)
+  const int rows = s.nch >= 2 ? (s.qr < 0 ? SONG_UNION_WIDE_ROWS : s.nch >= 4 ? SONG_XWIDE_ROWS : SONG_WIDE_ROWS)
                               : SONG_STAGE_ROWS;  // StageRows<NCH, UNION>::R
   const int stage_bytes = hamming ? 0 : SONG_STAGE_BUFS * rows * 512 * s.nch;  // Stage<NCH>::STRIDE
   const int cid_ints = steps > 1 ? 32 * song::MAX_STEPS : 32;  // located candidates
