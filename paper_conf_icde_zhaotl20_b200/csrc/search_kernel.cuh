@@ -747,6 +747,18 @@ struct Tier {
 #ifndef SONG_BULK_PF_NCH
 #define SONG_BULK_PF_NCH 2
 #endif
+// rows prefetched ahead for rows of >= SONG_PF_WINDOW_NCH chunks per lane
+// (32 = every later row at once).  GIST L 24 (1K queries x 10): window 32 /
+// 16 / 8 / 6 / 4 / 2 = 4.12 / 4.21 / 4.27 / 4.28 / 4.31 / 4.39 M QPS;
+// MNIST8m-shaped original vectors (25 GB, no reuse) at L 48: 1.11 M (32),
+// 1.32 M (8), 1.48 M (4), 1.49 M (2) — 1.47 M with 8-row rounds; the 1 KB /
+// 800 B rows of NYTimes / GloVe lose 0.5-2 % with a window (r03aq / r03ar A/B)
+#ifndef SONG_PF_WINDOW
+#define SONG_PF_WINDOW 2
+#endif
+#ifndef SONG_PF_WINDOW_NCH
+#define SONG_PF_WINDOW_NCH 8
+#endif
 #ifndef SONG_STAGE_BUFS
 #define SONG_STAGE_BUFS 1
 #endif
@@ -980,15 +992,23 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
   // 2.95 -> 3.27 M QPS with the bulk form, NYTimes' 1 KB rows 6.48 -> 6.69 M,
   // GloVe's 800 B rows unchanged, SIFT's 512 B rows 20.9 -> 19.9 M: kept
   // per line; profiles r03ah / r03ai A/B)
-  if (lane >= NBUF * R && lane < nc) {
-    const char* row = reinterpret_cast<const char*>(data) + (uint64_t)myid * rowbytes;
-    if (SONG_L2_PREFETCH == 1 || NCH >= SONG_BULK_PF_NCH) {
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(row), "r"(rowbytes) : "memory");
-    } else {
-      for (uint32_t o = 0; o < rowbytes; o += 128)
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(row + o));
+  // Rows of >= 8 chunks per lane keep at most SONG_PF_WINDOW rows prefetched
+  // ahead of the staged rounds (a rolling window, advanced one round at a
+  // time below): prefetching every later row at once overflows L2 when the
+  // rows have no reuse (MNIST8m-shaped 25 GB index).
+  constexpr int PFW = NCH >= SONG_PF_WINDOW_NCH ? SONG_PF_WINDOW : 32;
+  auto prefetch_rows = [&](int lo, int hi) {  // lanes lo <= lane < hi prefetch their row
+    if (lane >= lo && lane < hi && lane < nc) {
+      const char* row = reinterpret_cast<const char*>(data) + (uint64_t)myid * rowbytes;
+      if (SONG_L2_PREFETCH == 1 || NCH >= SONG_BULK_PF_NCH) {
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(row), "r"(rowbytes) : "memory");
+      } else {
+        for (uint32_t o = 0; o < rowbytes; o += 128)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(row + o));
+      }
     }
-  }
+  };
+  prefetch_rows(NBUF * R, NBUF * R + PFW);
 #endif
   for (int k = 0; k < rounds; ++k) {
     const int b = k * R;
@@ -1016,6 +1036,10 @@ __device__ __forceinline__ float bulk_distance(const float* __restrict__ data, i
     }
     // buffer k % NBUF is free again (this lane read only its own slices)
     if (k + NBUF < rounds) issue(k + NBUF);
+#if SONG_L2_PREFETCH
+    if (PFW < 32 && (k + NBUF + 1) * R + PFW - R < nc)  // slide the window by one round
+      prefetch_rows((k + NBUF) * R + PFW, (k + NBUF + 1) * R + PFW);
+#endif
     const float tot = transpose_reduce<R>(part, lane);
     const float got = __shfl_sync(FULL, tot, ((lane - b) & (R - 1)) << (5 - LR));
     if (lane >= b && lane < b + R) mine = got;
