@@ -132,8 +132,8 @@ typedef struct song_search_params {
                               batch order. */
   int32_t queue_kind;      /* how q and topk are held (results never depend on it).
                               SONG_QUEUE_AUTO (0, default): with visited HASH and steps
-                              <= 1 the bounded union (W in 1, 2 or 4 registers per lane
-                              for queue_len <= 128, in shared memory above); otherwise
+                              <= 1 the bounded union (W in 1, 2, 4 or 8 registers per
+                              lane for queue_len <= 256, in shared memory above); otherwise
                               separate q and topk, in registers for queue_len <= 128,
                               in shared memory above.
                               SONG_QUEUE_SEPARATE: q and topk as the paper keeps them

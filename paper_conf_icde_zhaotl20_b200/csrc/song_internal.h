@@ -57,9 +57,11 @@ struct song_index {
 };
 
 // the bounded union (reading R17) keeps W in registers up to this queue_len
-// (128: 4 u64 per lane; 256: 8), in shared-memory tiers above
+// (128: 4 u64 per lane; 256: 8), in shared-memory tiers above.  256: GloVe-IP
+// at L 160 1.61 -> 1.63 M QPS once the wide-row prefetches were bulk (r03ap;
+// 1.61 -> 1.56 M before, r03u)
 #ifndef SONG_RUN_MAX_L
-#define SONG_RUN_MAX_L 128
+#define SONG_RUN_MAX_L 256
 #endif
 
 namespace song {

@@ -61,10 +61,10 @@ def test_argument_errors_need_no_gpu():
 def test_union_is_the_default_queue():
     """Reading R17 (one bounded list W of q and topk) is what the library runs
     by default with the hash visited set and one pop per iteration: in
-    registers up to queue_len 128, in shared-memory tiers above; the paper's
+    registers up to queue_len 256, in shared-memory tiers above; the paper's
     separate q / topk on request, and for the other visited kinds."""
     from paper_conf_icde_zhaotl20_b200 import song
-    for L, regs in ((16, 1), (33, 2), (100, 4), (128, 4), (160, 0), (1280, 0)):
+    for L, regs in ((16, 1), (33, 2), (100, 4), (128, 4), (160, 8), (256, 8), (257, 0), (1280, 0)):
         pl = song.plan(song.Params(K=10, queue_len=L), 128)
         assert (pl.queue_kind, pl.queue_regs) == (2, regs), L
     sep = song.plan(song.Params(K=10, queue_len=64, queue_kind="separate"), 128)
@@ -143,7 +143,7 @@ def test_plan_lazy_capacity_bounds(L):
     p = song.plan(song.Params(K=1, queue_len=L), 128)
     slots = 1 << p.visited_log2
     assert 2 * L + 32 <= p.visited_cap <= 3 * slots // 4
-    assert p.queue_regs == (1 if L <= 32 else 2 if L <= 64 else 4 if L <= 128 else 0)
+    assert p.queue_regs == (1 if L <= 32 else 2 if L <= 64 else 4 if L <= 128 else 8 if L <= 256 else 0)
     assert p.smem_per_warp * p.warps_per_block <= 227 * 1024
     # eager deletion and multi-step probing report -1; other kinds 0
     assert song.plan(song.Params(K=1, queue_len=L, visited_cap=-1), 128).visited_cap == -1
