@@ -509,11 +509,23 @@ struct RegArr {
     for (int r = 0; r < QR; ++r) v[r] = KEY_MAX;
   }
   // element e (warp-uniform)
+  // (mask-and-or over every register, not a select chain: nvcc turns a chain
+  // keyed on a runtime index into an indexed local-memory access, which puts
+  // the whole array on the stack)
+  // (8 registers: the select chain, i.e. W indexed in local memory, measured
+  // faster than 8 masked ORs per access — GloVe-IP L 160 1.63 vs 1.52 M QPS;
+  // 2 / 4 registers: the masks — K = 100 6.11 -> 6.27 M, NYTimes 6.74 -> 6.91 M)
   __device__ __forceinline__ uint64_t get(int e) const {
-    uint64_t x = v[0];
+    uint64_t x = 0;
+    if constexpr (QR >= 8) {
+      x = v[0];
 #pragma unroll
-    for (int r = 1; r < QR; ++r)
-      if ((e >> 5) == r) x = v[r];
+      for (int r = 1; r < QR; ++r)
+        if ((e >> 5) == r) x = v[r];
+    } else {
+#pragma unroll
+      for (int r = 0; r < QR; ++r) x |= v[r] & (0ull - (uint64_t)((e >> 5) == r));
+    }
     return __shfl_sync(FULL, x, e & 31);
   }
   // remove element 0 (the head), shifting the rest down
@@ -1175,10 +1187,14 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 #ifndef SONG_RUN_LB_BLOCKS
 #define SONG_RUN_LB_BLOCKS 7
 #endif
+#ifndef SONG_RUN8_LB_BLOCKS  // W in 8 registers (queue_len 129-256)
+#define SONG_RUN8_LB_BLOCKS 7
+#endif
 template <int NCH, int QR = 1>
 struct MinBlocks {
   static constexpr int value =
-      NCH >= 4 ? SONG_XWIDE_LB_BLOCKS : (QR == 0 ? 5 : QR > 8 ? SONG_RUN_LB_BLOCKS : SONG_LB_BLOCKS);
+      NCH >= 4 ? SONG_XWIDE_LB_BLOCKS
+               : (QR == 0 ? 5 : QR == 16 ? SONG_RUN8_LB_BLOCKS : QR > 8 ? SONG_RUN_LB_BLOCKS : SONG_LB_BLOCKS);
 };
 // MS: multi-step probing (a.steps pops per iteration, <= MAX_STEPS; §V)
 constexpr int MAX_STEPS = 4;
@@ -1433,8 +1449,13 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
         q.pop_front(lane);
       } else if (RUN) {  // now moves from "q" to "topk" inside W
 #pragma unroll
-        for (int r = 0; r < QRr; ++r)
-          if ((wpos >> 5) == r && lane == (wpos & 31)) q.v[r] |= 1ull;
+        for (int r = 0; r < QRr; ++r) {  // (branch-free below 8 registers: see RegArr::get)
+          if constexpr (QRr >= 8) {
+            if ((wpos >> 5) == r && lane == (wpos & 31)) q.v[r] |= 1ull;
+          } else {
+            q.v[r] |= (uint64_t)(((wpos >> 5) == r) & (lane == (wpos & 31)));
+          }
+        }
       } else if (UNQ) {
         qg.set_flag(hint, lane);  // now moves from "q" to "topk" inside W
         hint = qg.next_unpopped(hint + 1, lane);
