@@ -66,7 +66,7 @@ def main():
                    "qps": round(b / (t / 1e3), 1)}
             log(json.dumps(row))
             rows.append(row)
-    res = {"figure": "Fig. 11 (P:1593-1631) on B200", "workload": "sift1m-shaped, R16 graph",
+    res = {"figure": "Fig. 11 (P:1593-1631) on B200", "workload": f"sift1m-shaped, {bench.GRAPH_DESC[bench.default_graph(cfg)]}",
            "rows": rows}
     line = json.dumps(res)
     print(line)
