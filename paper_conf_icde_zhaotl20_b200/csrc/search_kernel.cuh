@@ -1177,6 +1177,13 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 // union in registers: up to this many selected keys are inserted one at a
 // time (measured 0 / 2 / 4: SIFT L 16 20.75 / 21.01 / 20.87 M QPS, K = 100
 // 6.02 / 6.06 / 6.06 M, NYTimes 6.47 / 6.49 / 6.51 M; profiles r03ae A/B)
+// the union in registers reuses the locate probe's empty slot for the insert
+// of every candidate (lazy deletion: no tombstones, so the same slots a probe
+// would take): K = 100 6.23 -> 6.36 M QPS, NYTimes +0.8 %, SIFT L 16 +0.2 %
+// (r03be A/B, bit-exact)
+#ifndef SONG_SLOT_REUSE
+#define SONG_SLOT_REUSE 1
+#endif
 #ifndef SONG_RUN_INS_MAX
 #define SONG_RUN_INS_MAX 2
 #endif
@@ -1213,6 +1220,9 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   constexpr bool UNI = UNQ || RUN;  // R17 semantics (either storage)
   constexpr bool REG = QR > 0 && !RUN;  // separate q / topk in registers
   constexpr bool GVT = QR == -2;  // R17 with the visited table in global memory
+  // the locate probe hands each candidate's insert slot to the insert (the
+  // global tables; the union in registers with SONG_SLOT_REUSE)
+  constexpr bool SLOT = GVT || (RUN && SONG_SLOT_REUSE && VK == VK_HASH);
   constexpr int QRr = RUN ? QR - 8 : QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
@@ -1232,7 +1242,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   // (the evicted-key list only for the Cuckoo filter, the insert slots only
   // for GVT: the other kernels give those bytes to more resident warps)
   int* cslot = reinterpret_cast<int*>(ev + (VK == VK_CUCKOO ? 32 : 0));  // GVT: each candidate's insert slot
-  uint64_t* qa = reinterpret_cast<uint64_t*>(cslot + (GVT ? 32 : 0));  // q (or W, R17)
+  uint64_t* qa = reinterpret_cast<uint64_t*>(cslot + (SLOT ? 32 : 0));  // q (or W, R17)
   uint64_t* tk = qa + tslots;                   // topk (QR == 0 only)
   const int tkslots = QR == 0 ? tslots : 0;
   int* table = GVT ? a.gvis + ((size_t)blockIdx.x * (blockDim.x >> 5) + warp) * ((size_t)1 << a.table_log2)
@@ -1502,7 +1512,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       // (called by every lane: the probe loops are warp-collective)
       int eslot = -1;
       bool seen;
-      if constexpr (GVT)  // remember where each candidate's insert goes (one L2 trip less)
+      if constexpr (SLOT)  // remember where each candidate's insert goes (one probe less)
         seen = hs.contains_slot(v, keep, eslot);
       else
         seen = v_contains(v, keep);
@@ -1510,7 +1520,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
       const unsigned km = __ballot_sync(FULL, keep);
       int nc_all = __popc(km);
       if (keep) cid[__popc(km & lt)] = v;
-      if (GVT && keep) cslot[__popc(km & lt)] = eslot;
+      if (SLOT && keep) cslot[__popc(km & lt)] = eslot;
       __syncwarp();
       if constexpr (MS) {
         // the other popped rows, in pop order: one candidate list (R13)
@@ -1643,7 +1653,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
             used = RUN ? qsize : UNQ ? qg.size : na_g + tsize;
             __syncwarp();
           }
-          if (GVT && a.lazy && !rebuilt) {
+          if (SLOT && a.lazy && !rebuilt) {
             // the locate probe left each candidate's slot (the first EMPTY of
             // the bucket its probe ended in): one plain store per candidate,
             // the lowest lane of a shared slot wins, the others probe again
