@@ -1180,7 +1180,8 @@ __device__ __forceinline__ float dist_of(const float* __restrict__ data, int dpa
 // the union in registers reuses the locate probe's empty slot for the insert
 // of every candidate (lazy deletion: no tombstones, so the same slots a probe
 // would take): K = 100 6.23 -> 6.36 M QPS, NYTimes +0.8 %, SIFT L 16 +0.2 %
-// (r03be A/B, bit-exact)
+// (r03be A/B, bit-exact); W in 8 registers keeps the probing insert (GloVe-IP
+// L 160 1.63 vs 1.56 M, r03bg)
 #ifndef SONG_SLOT_REUSE
 #define SONG_SLOT_REUSE 1
 #endif
@@ -1222,7 +1223,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   constexpr bool GVT = QR == -2;  // R17 with the visited table in global memory
   // the locate probe hands each candidate's insert slot to the insert (the
   // global tables; the union in registers with SONG_SLOT_REUSE)
-  constexpr bool SLOT = GVT || (RUN && SONG_SLOT_REUSE && VK == VK_HASH);
+  constexpr bool SLOT = GVT || (RUN && QRr <= 4 && SONG_SLOT_REUSE && VK == VK_HASH);
   constexpr int QRr = RUN ? QR - 8 : QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;

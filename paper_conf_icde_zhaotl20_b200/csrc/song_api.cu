@@ -350,7 +350,7 @@ Shape search_shape(int L, int vk, const song_search_params* p, int dpad, bool ha
   // [32 insert slots: the union with global tables, added below], tiers, table
   s.warp_bytes = stage_bytes + qsm_bytes + 16 + cid_ints * 4 + 32 * 8 +
                  (vk == song::VK_CUCKOO ? 32 * 8 : 0) +
-                 (SONG_SLOT_REUSE && s.qr > 8 && vk == song::VK_HASH ? 32 * 4 : 0) +
+                 (SONG_SLOT_REUSE && s.qr > 8 && s.qr < 16 && vk == song::VK_HASH ? 32 * 4 : 0) +
                  (s.qr <= 0 ? (s.qr == 0 ? 2 : 1) * (((L + 63) / 64) * 64) * 8 + 8 : 0) +
                  tbytes;
   s.warp_bytes = (s.warp_bytes + 127) & ~127;
