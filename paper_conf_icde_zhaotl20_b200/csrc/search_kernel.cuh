@@ -1223,7 +1223,7 @@ __global__ void __launch_bounds__(SONG_LB_THREADS, MinBlocks<NCH, QR>::value)
   constexpr bool GVT = QR == -2;  // R17 with the visited table in global memory
   // the locate probe hands each candidate's insert slot to the insert (the
   // global tables; the union in registers with SONG_SLOT_REUSE)
-  constexpr bool SLOT = GVT || (RUN && QRr <= 4 && SONG_SLOT_REUSE && VK == VK_HASH);
+  constexpr bool SLOT = GVT || (RUN && QR < 16 && SONG_SLOT_REUSE && VK == VK_HASH);
   constexpr int QRr = RUN ? QR - 8 : QR > 0 ? QR : 1;
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
